@@ -1,0 +1,418 @@
+#!/usr/bin/env python
+"""Benchmark of the fused relational hot path on B200 (one JSON line on rank 0).
+
+Headline (BASELINE.json configs[1]): fused back-to-back SELECTs (k=2, s=0.5
+per stage) over 2^28 device-resident int32 rows per GPU; a step is
+one fused select_chain kernel (+ at N>1 the NCCL all_gather of the per-rank
+counts and the exclusive scan into global output offsets).
+`value` = rows/s over all ranks (weak scaling: 2^28 rows per rank).
+
+The same line carries
+  roofline      select_fused kernel: algorithmic bytes (4 B in + 4 B per kept
+                row out) / mean kernel time vs MEASURED_PEAKS.json hbm_gbs
+  e2e           the same chain through ra_fission_run from pinned HOST buffers
+                (H2D + D2H inside the timed region), rows/s
+  cpu_baseline  the CPU oracle (single thread, as it stands) on the same data
+  q1_sf10 / q1_sf100 / select_1m / unfused / sweep  the other BASELINE configs
+  clocks        SM clocks and throttle reasons sampled during the timed region
+
+`--impl reference` runs the CPU oracle as the reference arm on the same config.
+Launch: python bench.py [--gpus N --steps K --warmup W]; N>1 under torchrun.
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import ragen  # noqa: E402  (input generator: no method arithmetic)
+
+METRIC = "rows/s (fused SELECT chain k=2 s=0.5, 2^28 int32 rows/GPU, device-resident)"
+CHAIN_SEED, Q1_SEED, D1_SEED = 2, 5, 1
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--rows-log2", type=int, default=28)
+    ap.add_argument("--k", type=int, default=2)
+    ap.add_argument("--sel", type=float, default=0.5)
+    ap.add_argument("--no-extras", action="store_true", help="headline only (for ncu runs)")
+    ap.add_argument("--sweep", action="store_true", help="selectivity x k sweep, fused vs unfused")
+    ap.add_argument("--fission-sweep", action="store_true")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- plumbing
+class Dist:
+    def __init__(self):
+        self.world = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.local = int(os.environ.get("LOCAL_RANK", "0"))
+        self.pg = None
+
+    def init(self, torch):
+        if self.world > 1:
+            import torch.distributed as dist
+            dist.init_process_group("nccl", device_id=torch.device("cuda", self.local))
+            self.pg = dist
+
+    def barrier(self, torch):
+        if self.pg:
+            self.pg.barrier()
+        torch.cuda.synchronize()
+
+    def max(self, torch, v: float) -> float:
+        if not self.pg:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device="cuda")
+        self.pg.all_reduce(t, op=self.pg.ReduceOp.MAX)
+        return float(t.item())
+
+
+class ClockSampler:
+    """nvidia-smi-equivalent clocks/throttle sampling (NVML) during a region."""
+
+    REASONS = {
+        0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+        0x20: "sw_thermal_slowdown", 0x4: "sw_power_cap", 0x1: "gpu_idle", 0x2: "applications_clocks_setting",
+    }
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover
+            self.nv = None
+            self.err = str(e)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        if not self.nv:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(key: str):
+    """dram bytes per launch from the committed ncu --set full capture, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f).get(key)
+    return None
+
+
+def timed(torch, D: Dist, fn, steps: int, warmup: int, kernel_fn=None):
+    """W warm-up steps; then EXACTLY `steps` steps between barrier+sync on both
+    sides, CUDA events on the launching (current) stream; max over ranks.
+    Returns (ms_per_step, mean kernel ms or None)."""
+    for i in range(warmup):
+        fn(i)
+    D.barrier(torch)
+    s = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)] \
+        if kernel_fn else None
+    e0.record(s)
+    for i in range(steps):
+        if kev:
+            kev[i][0].record(s)
+            kernel_fn(i)
+            kev[i][1].record(s)
+            fn(i, kernel_done=True)
+        else:
+            fn(i)
+    e1.record(s)
+    e1.synchronize()
+    D.barrier(torch)
+    ms = e0.elapsed_time(e1) / steps
+    kms = statistics.mean(a.elapsed_time(b) for a, b in kev) if kev else None
+    ms = D.max(torch, ms)
+    if kms is not None:
+        kms = D.max(torch, kms)
+    return ms, kms
+
+
+# ---------------------------------------------------------------- our arm
+def run_ours(args, D: Dist):
+    import torch
+    D.init(torch)
+    torch.cuda.set_device(D.local)
+    import paper_conf_ipps_wudwcyc12_b200 as R
+
+    dev = torch.device("cuda", D.local)
+    stream = torch.cuda.current_stream()
+    sh = int(stream.cuda_stream)
+    n = 1 << args.rows_log2
+    k, s_sel = args.k, args.sel
+    thresholds = ragen.nested_thresholds(s_sel, k)
+    preds = [("lt", t) for t in thresholds]
+    P = R.make_preds(preds)
+
+    # rank r owns global rows [r*n, (r+1)*n) of one seeded column (weak scaling)
+    x = torch.empty(n, dtype=torch.int32, device=dev)
+    ragen.int32_column_dev(CHAIN_SEED, x, row0=D.rank * n, stream=sh)
+    out = torch.empty(n, dtype=torch.int32, device=dev)
+    cnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    ws_bytes = R.ra_select_workspace_bytes(n, k, 1)
+    ws = torch.zeros(ws_bytes, dtype=torch.uint8, device=dev)
+    counts_all = torch.zeros(D.world, dtype=torch.int64, device=dev)
+    offsets = torch.zeros(D.world, dtype=torch.int64, device=dev)
+    args_chain = (x.data_ptr(), n, P, k, 1, out.data_ptr(), n, cnt.data_ptr(), ws.data_ptr(), ws_bytes, sh)
+
+    def chain_kernel(i):
+        R.ra_select_chain(*args_chain)
+
+    def chain_step(i, kernel_done=False):
+        if not kernel_done:
+            chain_kernel(i)
+        if D.pg:  # a9: gather per-rank counts -> exclusive scan -> global offsets
+            D.pg.all_gather_into_tensor(counts_all, cnt)
+            torch.cumsum(counts_all, 0, out=offsets)
+
+    torch.cuda.synchronize()
+    launches0 = R.ra_kernel_launches()
+    with ClockSampler(D.local) as clk:
+        ms, kms = timed(torch, D, chain_step, args.steps, args.warmup, kernel_fn=chain_kernel)
+    launches = R.ra_kernel_launches() - launches0 - args.warmup
+    kept = int(cnt.item())
+    value = D.world * n / (ms * 1e-3)
+    peak, peak_src = peaks()
+    alg_bytes = 4 * n + 4 * kept
+    achieved = alg_bytes / (kms * 1e-3) / 1e9
+    res = {
+        "metric": METRIC, "value": value, "unit": "rows/s", "n_gpus": D.world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "int32", "data": "synthetic (seeded uniform int32, ragen)",
+        "config": {"workload": f"configs[1]: fused {k}x SELECT, s={s_sel}/stage, 2^{args.rows_log2} int32 rows/GPU, device-resident",
+                   "rows_per_gpu": n, "k": k, "sel_per_stage": s_sel, "kept_per_gpu": kept,
+                   "l2": "inputs > L2 (1 GiB column per step vs 126 MB L2), no flush needed",
+                   "parallelism": f"row-range shards x{D.world}, NCCL all_gather of counts"},
+        "gpu_launches": launches,
+        "roofline": {"kernel": "select_fused_kernel", "bound": "hbm", "achieved": achieved, "peak": peak,
+                     "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": ncu_traffic(f"select_fused_k{k}_s{s_sel}_n{args.rows_log2}"),
+                     "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kms},
+        "clocks": clk.summary(),
+    }
+    if not args.no_extras:
+        res.update(extras(args, D, torch, R, x, preds, kept, ms))
+    if D.rank == 0:
+        print(json.dumps(res), flush=True)
+
+
+def extras(args, D, torch, R, x, preds, kept, chain_ms):
+    """Other BASELINE configs + e2e + CPU baseline, same timing rules."""
+    dev = x.device
+    sh = int(torch.cuda.current_stream().cuda_stream)
+    n = x.numel()
+    k = len(preds)
+    peak, _ = peaks()
+    ex = {}
+
+    # --- unfused composition of the same chain (the paper's "without round trip")
+    if k > 1:
+        uo = torch.empty(n, dtype=torch.int32, device=dev)
+        uc = torch.zeros(1, dtype=torch.int64, device=dev)
+        uws_b = R.ra_select_workspace_bytes(n, k, 0)
+        uws = torch.zeros(uws_b, dtype=torch.uint8, device=dev)
+        P = R.make_preds(preds)
+        a = (x.data_ptr(), n, P, k, 0, uo.data_ptr(), n, uc.data_ptr(), uws.data_ptr(), uws_b, sh)
+        ums, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_chain(*a), 20, 3)
+        assert int(uc.item()) == kept
+        ex["unfused"] = {"rows_per_s": D.world * n / (ums * 1e-3), "ms_per_step": ums,
+                         "fused_over_unfused": ums / chain_ms, "launches_per_step": k}
+        del uo, uws
+
+    # --- e2e: same chain from pinned host memory through ra_fission_run
+    if D.rank == 0 or True:
+        h_in = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        h_in.copy_(x.cpu())
+        h_out = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        chunk = 1 << 24
+        streams = [torch.cuda.Stream() for _ in range(3)]
+        h_counts = torch.zeros((n + chunk - 1) // chunk, dtype=torch.int64, pin_memory=True)
+        R.fission_run(h_in, preds, chunk, streams, h_out=h_out, h_chunk_counts=h_counts)
+        D.barrier(torch)
+        t0 = time.perf_counter()
+        reps = 3
+        for _ in range(reps):
+            _, c = R.fission_run(h_in, preds, chunk, streams, h_out=h_out, h_chunk_counts=h_counts)
+        dt = (time.perf_counter() - t0) / reps
+        dt = D.max(torch, dt)
+        assert c == kept
+        ex["e2e"] = {"value": D.world * n / dt, "unit": "rows/s", "h2d_bytes_per_step": 4 * n,
+                     "d2h_bytes_per_step": 4 * c + 8 * h_counts.numel(), "ms_per_step": dt * 1e3,
+                     "path": "ra_fission_run: pinned host in/out, chunk 2^24 rows, 3 streams (fusion+fission)",
+                     "pcie_h2d_gbs": 4 * n / dt / 1e9}
+        del h_in, h_out
+
+    # --- configs[0]: single SELECT on 2^20 rows, 50% (latency-bound, L2-resident)
+    n1 = 1 << 20
+    x1 = torch.empty(n1, dtype=torch.int32, device=dev)
+    ragen.int32_column_dev(D1_SEED, x1, stream=sh)
+    o1 = torch.empty(n1, dtype=torch.int32, device=dev)
+    c1 = torch.zeros(1, dtype=torch.int64, device=dev)
+    ws1_b = R.ra_select_workspace_bytes(n1, 1, 1)
+    ws1 = torch.zeros(ws1_b, dtype=torch.uint8, device=dev)
+    P1 = R.make_preds([("lt", 0)])
+    a1 = (x1.data_ptr(), n1, P1, 1, 1, o1.data_ptr(), n1, c1.data_ptr(), ws1.data_ptr(), ws1_b, sh)
+    ms1, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_chain(*a1), 200, 10)
+    ex["select_1m"] = {"us_per_call": ms1 * 1e3, "rows_per_s": n1 / (ms1 * 1e-3), "kept": int(c1.item()),
+                       "note": "configs[0]; 6 MiB L2-resident, back-to-back stream launches"}
+
+    # --- configs[2]: Q1 SF10 device-resident (N=1 only) and configs[4] SF100 sharded
+    def q1_bench(sf, shard):
+        N = ragen.rows_for_sf(sf)
+        lo, hi = (D.rank * N // D.world, (D.rank + 1) * N // D.world) if shard else (0, N)
+        m = hi - lo
+        cols = {name: torch.empty(m, dtype=getattr(torch, np.dtype(dt).name), device=dev)
+                for name, dt in ragen.LINEITEM_COLUMNS}
+        ragen.lineitem_dev(Q1_SEED, ragen.parts_for_sf(sf), cols, row0=lo, stream=sh)
+        part = torch.zeros(ctypes.sizeof(R.ra_q1_partial), dtype=torch.uint8, device=dev)
+        wsq_b = R.ra_q1_workspace_bytes(m)
+        wsq = torch.zeros(wsq_b, dtype=torch.uint8, device=dev)
+        li = R.lineitem_struct(cols)
+        parts = torch.zeros(D.world * part.numel(), dtype=torch.uint8, device=dev)
+
+        def kern(i):
+            R.ra_q1(li, m, R.Q1_CUTOFF_DELTA90, part.data_ptr(), wsq.data_ptr(), wsq_b, sh)
+
+        def step(i, kernel_done=False):
+            if not kernel_done:
+                kern(i)
+            if D.pg and shard:
+                D.pg.all_gather_into_tensor(parts, part)
+
+        qms, qkms = timed(torch, D, step, 50, 5, kernel_fn=kern)
+        raw = (parts if (D.pg and shard) else part).cpu().numpy().tobytes()
+        rows, rc = R.q1_finalize(raw)
+        ach = 38 * m / (qkms * 1e-3) / 1e9
+        del cols
+        return {"rows": N, "rows_per_s": (N if shard else m) / (qms * 1e-3), "ms_per_step": qms,
+                "kernel_ms": qkms, "groups": len(rows), "finalize_rc": rc,
+                "roofline": {"kernel": "q1_fused_kernel", "bound": "hbm", "achieved": ach, "peak": peak,
+                             "unit": "GB/s", "frac": ach / peak, "algorithmic_bytes_per_launch": 38 * m,
+                             "traffic": ncu_traffic(f"q1_sf{int(sf)}")}}
+
+    if D.world == 1:
+        ex["q1_sf10"] = q1_bench(10, False)
+    ex["q1_sf100"] = q1_bench(100, True)
+    ex["q1_sf100"]["scaling"] = "strong (600M rows split over ranks)"
+
+    # --- CPU baseline: the oracle as it stands, rank 0, N=1 only
+    if D.world == 1 and D.rank == 0:
+        ex["cpu_baseline"] = cpu_baseline(x, preds, n)
+    return ex
+
+
+def cpu_baseline(x, preds, n):
+    import oracle  # test infrastructure: only this leg of bench.py may use it
+    sample = min(n, 1 << 26)
+    xh = x[:sample].cpu().numpy()
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        c = oracle.select(xh, preds).size
+        reps += 1
+        if time.perf_counter() - t0 > 2.0:
+            break
+    dt = (time.perf_counter() - t0) / reps
+    return {"value": sample / dt, "unit": "rows/s", "cores": 1, "kind": "oracle",
+            "sample": f"first 2^{sample.bit_length() - 1} rows of the same column, oracle_select (C, -O2, 1 thread)",
+            "kept": c}
+
+
+# ---------------------------------------------------------- reference arm
+def run_reference(args, D: Dist):
+    """The CPU oracle as the reference arm, same config/metric/unit."""
+    if D.rank != 0:
+        return
+    import oracle
+    n = 1 << args.rows_log2
+    sample = min(n, 1 << 24)
+    x = ragen.int32_column(CHAIN_SEED, sample)
+    preds = [("lt", t) for t in ragen.nested_thresholds(args.sel, args.k)]
+    for _ in range(max(1, args.warmup)):
+        oracle.select(x, preds)
+    steps = max(1, min(args.steps, 20))
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        out = oracle.select(x, preds)
+    dt = (time.perf_counter() - t0) / steps
+    v = sample / dt
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "rows/s", "n_gpus": args.gpus,
+        "steps": steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic (seeded uniform int32, ragen)",
+        "config": {"workload": f"configs[1]: fused {args.k}x SELECT, s={args.sel}/stage, 2^{args.rows_log2} int32 rows; "
+                               f"oracle step = bounded sample of 2^24 rows", "kept": int(out.size)},
+        "cpu_baseline": {"value": v, "unit": "rows/s", "cores": 1, "kind": "oracle",
+                         "sample": "2^24 rows of the configs[1] column per step (plain C oracle, 1 thread)"},
+        "e2e": {"value": v, "unit": "rows/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    args = parse()
+    D = Dist()
+    if args.impl == "reference":
+        run_reference(args, D)
+        return
+    run_ours(args, D)
+    if D.pg:
+        D.pg.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,233 @@
+/* ra.h — C ABI of libra.so: the fused relational-operator hot path of
+ * Wu, Diamos, Wang, Cadambi, Yalamanchili, Chakradhar, "Optimizing Data
+ * Warehousing Applications for GPUs Using Kernel Fusion/Fission" (IPDPSW 2012),
+ * built B200-native (sm_100a).
+ *
+ * Citations are PAPER.md line numbers with the section/figure/table they sit
+ * in; "SURVEY Cn" = the reading of the paper recorded in SURVEY.md §8(c) and
+ * DESIGN.md; EXT:TPC-H = the TPC-H specification (paper ref [9], L1791-1792).
+ *
+ * Conventions for every entry point
+ *  - Plain pointers and sizes only.  "d_" = device pointer, "h_" = host pointer.
+ *    All buffers are caller-owned; the library never allocates device memory.
+ *  - Stream-ordered entry points (ra_select, ra_select_chain, ra_q1) enqueue
+ *    work on `stream` and return immediately; results are valid once the
+ *    caller synchronises that stream.  ra_fission_run and ra_q1_finalize are
+ *    synchronous.
+ *  - Return value: RA_OK or a negative RA_E_* code; nothing is enqueued when
+ *    an argument check fails.  ra_last_error() gives a thread-local message.
+ *    No exception or abort crosses the ABI.
+ *  - Calls are reentrant given distinct workspaces; a workspace may be reused
+ *    by successive calls ordered on one stream.
+ *  - Workspaces must be zero-filled once after allocation (ra_workspace_init
+ *    or any memset); the library keeps them self-cleaning afterwards.
+ */
+#ifndef RA_H
+#define RA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Same type as cudaStream_t / CUstream; NULL = the legacy default stream. */
+typedef struct CUstream_st* ra_stream_t;
+
+/* ------------------------------------------------------------ error codes */
+#define RA_OK 0
+#define RA_E_INVAL (-1)       /* null pointer with n > 0, bad op, k > RA_MAX_PREDS,
+                                 k < 0, n < 0, chunk_rows <= 0, misaligned pointer,
+                                 n >= 2^32 where a call bounds n */
+#define RA_E_CAPACITY (-2)    /* (synchronous calls) result larger than out_cap:
+                                 the first out_cap values are written and the
+                                 count output holds the full (required) count */
+#define RA_E_DOMAIN (-3)      /* ra_q1_finalize: a partial reported rows outside
+                                 the Q1 domain (see ra_q1_partial.status) */
+#define RA_E_NOT_PINNED (-4)  /* ra_fission_run: a host buffer is not page-locked */
+#define RA_E_CUDA (-5)        /* a CUDA runtime call failed (message has details) */
+#define RA_E_WORKSPACE (-6)   /* ws_bytes smaller than the *_workspace_bytes size */
+
+/* Thread-local message describing the last non-RA_OK return on this thread. */
+const char* ra_last_error(void);
+
+/* ABI version (bumped on any layout change). */
+int ra_version(void);
+
+/* Number of CUDA kernels this process has launched through libra.so
+ * (monotonic; used by bench.py to report gpu_launches). */
+uint64_t ra_kernel_launches(void);
+
+/* Zero-fill a workspace (cudaMemsetAsync).  Needed once after allocation. */
+int ra_workspace_init(void* d_ws, size_t ws_bytes, ra_stream_t stream);
+
+/* ================================================================ SELECT
+ * Predicate: the element compared with a constant, signed int32 —
+ * "d < THRESHOLD" (Table III, §III-A) and "field.0==2" (Table I,
+ * L153-156); SURVEY C1.  A chain is the conjunction of its predicates
+ * (back-to-back SELECTs, Fig 2(a)).
+ */
+#define RA_MAX_PREDS 8
+enum { RA_LT = 0, RA_LE = 1, RA_GT = 2, RA_GE = 3, RA_EQ = 4, RA_NE = 5 };
+
+typedef struct {
+  int32_t op;    /* RA_LT .. RA_NE */
+  int32_t value; /* the constant */
+} ra_pred;
+
+/* Device workspace needed by ra_select / ra_select_chain for n rows.
+ * fused != 0: one pass (tile status words only, ~2*8*n/4096 B + 256 B).
+ * fused == 0: the unfused composition also keeps two intermediate int32[n]
+ * relations on the device ("without round trip", L972-984). */
+size_t ra_select_workspace_bytes(int64_t n, int k, int fused);
+
+/* Single SELECT: d_out[0..count) = the elements of d_in[0..n) satisfying
+ * `pred`, in input order; *d_count = count (int64, device).
+ *
+ * The paper's four stages — partition, filter, buffer, gather (Fig 3,
+ * L303-310, L479-485) — run as ONE kernel: each CTA takes a 4096-row tile by
+ * atomic ticket (partition), evaluates the predicate in registers (filter),
+ * compacts matches in shared memory via warp ballots/scans (buffer) and
+ * obtains its global output offset by a decoupled look-back over the tile
+ * status words instead of the paper's global sync + second gather kernel
+ * (gather).  Output order is the input order.
+ *
+ *  d_in      int32[n], 4-byte aligned (any sub-view of a device buffer)
+ *  n         >= 0; n = 0 writes *d_count = 0
+ *  d_out     int32[out_cap], 4-byte aligned; if count > out_cap only the first
+ *            out_cap values are written, *d_count still holds the full count
+ *  d_count   int64, device
+ *  d_ws      workspace of ra_select_workspace_bytes(n, 1, 1) bytes (zeroed once)
+ */
+int ra_select(const int32_t* d_in, int64_t n, ra_pred pred, int32_t* d_out, int64_t out_cap,
+              int64_t* d_count, void* d_ws, size_t ws_bytes, ra_stream_t stream);
+
+/* Chain of k back-to-back SELECTs over one input (Fig 2(a), Fig 6).
+ *  h_preds   host array of k predicates, 0 <= k <= RA_MAX_PREDS; k = 0 copies
+ *  fused     != 0: one kernel evaluates all k predicates per element in
+ *            registers — one partition/buffer/gather for the chain (L784-785,
+ *            L812-814); the conjunction is simplified once on the host to an
+ *            interval plus != exclusions (the Table III compiler benefit,
+ *            L790-805).
+ *            == 0: the unfused composition — k single-predicate passes with
+ *            device-resident intermediates in d_ws (the paper's "without
+ *            round trip" baseline, L972-984).  Same output (L580-581).
+ * Other arguments as ra_select; ws sized by ra_select_workspace_bytes(n, k, fused).
+ */
+int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,
+                    int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                    size_t ws_bytes, ra_stream_t stream);
+
+/* ============================================================ TPC-H Q1
+ * SELECT (l_shipdate <= cutoff) -> PROJECT (disc_price = price*(1-disc),
+ * charge = disc_price*(1+tax)) -> GROUP BY (returnflag, linestatus)
+ * SUM/COUNT, in one kernel with private accumulators and no HBM
+ * intermediates (Fig 2(g)(h); Q1 plan §V; EXT:TPC-H;
+ * SURVEY C8-C13).  The plan's JOINs are identities in a positional column
+ * store and its SORT orders at most 6 groups (C9): neither is executed.
+ *
+ * Columns (SoA, device, n rows each; decimals are int64 fixed point x100, C10):
+ *  shipdate int32 days since 1970-01-01; returnflag/linestatus bytes;
+ *  quantity, extendedprice, discount, tax int64 x100.
+ * Domain (checked on the SELECTED rows; violations are reported through
+ * ra_q1_partial.status and such rows are not accumulated):
+ *  returnflag in {'A','N','R'}, linestatus in {'F','O'}        (status bit 0)
+ *  0 <= quantity, extendedprice < 2^31; 0 <= discount, tax <= 100 (status bit 1)
+ * n < 2^32 per call.  Pointers must be naturally aligned.
+ */
+#define RA_Q1_GROUPS 6 /* slot = 2*rf + ls, rf: A=0 N=1 R=2, ls: F=0 O=1 */
+
+typedef struct {
+  const int32_t* shipdate;
+  const uint8_t* returnflag;
+  const uint8_t* linestatus;
+  const int64_t* quantity;
+  const int64_t* extendedprice;
+  const int64_t* discount;
+  const int64_t* tax;
+} ra_lineitem;
+
+/* Exact per-group sums.  Scales: qty/price/disc x1e2, disc_price x1e4,
+ * charge x1e6; disc_price and charge are 128-bit (lo + hi<<64), C11. */
+typedef struct {
+  int64_t count;
+  int64_t sum_qty;
+  int64_t sum_base_price;
+  int64_t sum_disc;
+  uint64_t sum_disc_price_lo;
+  int64_t sum_disc_price_hi;
+  uint64_t sum_charge_lo;
+  int64_t sum_charge_hi;
+} ra_q1_group;
+
+/* One shard's partial aggregate; shards combine by exact slotwise addition. */
+typedef struct {
+  uint32_t status;   /* OR of domain bits over selected rows (0 = clean) */
+  uint32_t n_groups; /* RA_Q1_GROUPS */
+  uint64_t rows;     /* rows scanned */
+  ra_q1_group group[RA_Q1_GROUPS];
+} ra_q1_partial;
+
+/* One output row of Q1 (ORDER BY returnflag, linestatus). */
+typedef struct {
+  uint8_t returnflag, linestatus, _pad[6];
+  int64_t count_order;
+  int64_t sum_qty;        /* x1e2 */
+  int64_t sum_base_price; /* x1e2 */
+  int64_t sum_disc;       /* x1e2 */
+  uint64_t sum_disc_price_lo; /* x1e4, 128-bit */
+  int64_t sum_disc_price_hi;
+  uint64_t sum_charge_lo;     /* x1e6, 128-bit */
+  int64_t sum_charge_hi;
+  double avg_qty, avg_price, avg_disc; /* (double)sum / (double)(100*count), C12 */
+} ra_q1_row;
+
+size_t ra_q1_workspace_bytes(int64_t n);
+
+/* Enqueue the fused Q1 kernel.  h_cols: host struct of DEVICE column
+ * pointers; shipdate_cutoff inclusive (TPC-H DELTA=90: 10471 = 1998-09-02);
+ * d_partial: device ra_q1_partial written completely (all 6 slots). */
+int ra_q1(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff,
+          ra_q1_partial* d_partial, void* d_ws, size_t ws_bytes, ra_stream_t stream);
+
+/* Host: sum n_partials partials exactly (row-range shards, fission chunks),
+ * drop empty groups, order by (returnflag, linestatus), compute the AVGs
+ * ("Aggregate/Unique", Fig 17(a)).  h_rows holds >= 6 rows.
+ * Returns RA_E_DOMAIN (rows still filled) if any partial has status != 0. */
+int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h_rows,
+                   int* n_rows);
+
+/* ============================================================= FISSION
+ * Host-resident SELECT chain with kernel fission (§IV; pipelined
+ * segments §IV-B; fusion+fission §IV-C).
+ * The input is split into contiguous chunks of chunk_rows (last one shorter);
+ * chunk c runs on streams[c % n_streams]: H2D copy -> select_chain kernel ->
+ * D2H of exactly that chunk's count into h_out at the running offset (the
+ * paper's "CPU gather", L1466-1468).  Copies of one chunk overlap the kernel
+ * of another; time ~ max(H2D, compute, D2H) (L1504-1509).  Output equals
+ * ra_select_chain on the whole input (C16).  Synchronous.
+ *
+ *  h_in            pinned host int32[n]
+ *  h_preds, k      as ra_select_chain; fused selects the chain kernel form
+ *  chunk_rows      > 0 (chunk_rows >= n with one stream = the "serial" mode)
+ *  streams         n_streams >= 1 CUDA streams of the current device
+ *  h_out           pinned host int32[out_cap]
+ *  h_count         host int64: total selected (the required size if > out_cap)
+ *  h_chunk_counts  pinned host int64[ceil(n/chunk_rows)]: per-chunk counts,
+ *                  written by the device through its mapped alias
+ *  d_ws            ra_fission_workspace_bytes(chunk_rows, n_streams, k, fused)
+ * Returns RA_E_CAPACITY if the total exceeds out_cap (first out_cap written).
+ */
+size_t ra_fission_workspace_bytes(int64_t chunk_rows, int n_streams, int k, int fused);
+
+int ra_fission_run(const int32_t* h_in, int64_t n, const ra_pred* h_preds, int k, int fused,
+                   int64_t chunk_rows, const ra_stream_t* streams, int n_streams, int32_t* h_out,
+                   int64_t out_cap, int64_t* h_count, int64_t* h_chunk_counts, void* d_ws,
+                   size_t ws_bytes);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* RA_H */

@@ -1,0 +1,146 @@
+"""B200-native fused relational-operator hot path (Wu et al., IPDPSW 2012).
+
+The product is ``libra.so`` (C ABI in ``include/ra.h``): hand-written sm_100a
+kernels for the fused SELECT chain, fused TPC-H Q1 and the kernel-fission
+pipeline.  This package is the thin Python layer above it:
+
+* ``ra_*`` — one-to-one ctypes bindings of the C entry points (``_ra.py``);
+* ``select_chain``, ``q1``, ``q1_finalize``, ``fission_run`` — conveniences
+  that take torch tensors, allocate outputs/workspaces with torch (device
+  memory and streams are PyTorch's; nothing else is) and call the bindings.
+
+There is no CPU or PyTorch fallback: every step of the path runs in libra.so.
+"""
+from __future__ import annotations
+
+import ctypes
+
+from ._ra import *  # noqa: F401,F403
+from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, ra_fission_run,
+                  ra_fission_workspace_bytes, ra_lineitem, ra_q1, ra_q1_finalize, ra_q1_partial,
+                  ra_q1_row, ra_q1_workspace_bytes, ra_select_chain, ra_select_workspace_bytes)
+
+Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
+LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
+
+_WS: dict = {}
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream_handle(stream) -> int:
+    torch = _torch()
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return int(stream.cuda_stream) if hasattr(stream, "cuda_stream") else int(stream)
+
+
+def workspace(device, kind: str, nbytes: int, stream=None):
+    """Zero-initialised, cached per (device, kind, stream) workspace tensor."""
+    torch = _torch()
+    key = (str(device), kind, _stream_handle(stream))
+    ws = _WS.get(key)
+    if ws is None or ws.numel() < nbytes:
+        ws = torch.zeros(max(256, nbytes), dtype=torch.uint8, device=device)
+        _WS[key] = ws
+    return ws
+
+
+def select_chain(x, preds, fused: bool = True, out=None, count=None, stream=None):
+    """Fused (or unfused) SELECT chain over a CUDA int32 tensor.
+
+    Returns ``(out, count)``: ``out[:count]`` holds the selected values in
+    input order; ``count`` is a 1-element int64 CUDA tensor (not synchronised).
+    """
+    torch = _torch()
+    if not (x.is_cuda and x.dtype == torch.int32 and x.is_contiguous()):
+        raise ValueError("x must be a contiguous CUDA int32 tensor")
+    n, k = x.numel(), len(preds)
+    if out is None:
+        out = torch.empty(max(1, n), dtype=torch.int32, device=x.device)
+    if count is None:
+        count = torch.empty(1, dtype=torch.int64, device=x.device)
+    need = ra_select_workspace_bytes(n, k, int(fused))
+    ws = workspace(x.device, "select_fused" if fused else "select_unfused", need, stream)
+    P = make_preds(preds)
+    ra_select_chain(x.data_ptr(), n, P, k, int(fused), out.data_ptr(), out.numel(), count.data_ptr(),
+                    ws.data_ptr(), ws.numel(), _stream_handle(stream))
+    return out, count
+
+
+def lineitem_struct(cols) -> ra_lineitem:
+    return ra_lineitem(*[cols[name].data_ptr() for name in LINEITEM_COLUMNS])
+
+
+def q1(cols, cutoff: int = Q1_CUTOFF_DELTA90, partial=None, stream=None):
+    """Fused Q1 over CUDA lineitem columns; returns the device partial (uint8[400])."""
+    torch = _torch()
+    sd = cols["shipdate"]
+    n = sd.numel()
+    if partial is None:
+        partial = torch.empty(ctypes.sizeof(ra_q1_partial), dtype=torch.uint8, device=sd.device)
+    ws = workspace(sd.device, "q1", ra_q1_workspace_bytes(n), stream)
+    ra_q1(lineitem_struct(cols), n, int(cutoff), partial.data_ptr(), ws.data_ptr(), ws.numel(),
+          _stream_handle(stream))
+    return partial
+
+
+def partials_from_bytes(buf: bytes, n_partials: int = 1):
+    arr = (ra_q1_partial * n_partials)()
+    ctypes.memmove(arr, buf, ctypes.sizeof(arr))
+    return arr
+
+
+def q1_finalize(partials):
+    """Host finalize of one or more partials (ctypes array or bytes).
+
+    Returns ``(rows, rc)`` with rows as dicts (exact ints, AVG doubles) and
+    ``rc`` = RA_OK or RA_E_DOMAIN.
+    """
+    if isinstance(partials, (bytes, bytearray)):
+        partials = partials_from_bytes(bytes(partials), len(partials) // ctypes.sizeof(ra_q1_partial))
+    rows = (ra_q1_row * RA_Q1_GROUPS)()
+    nrows = ctypes.c_int(0)
+    rc = ra_q1_finalize(partials, len(partials), rows, ctypes.byref(nrows))
+    out = []
+    for r in rows[:nrows.value]:
+        out.append({
+            "returnflag": chr(r.returnflag), "linestatus": chr(r.linestatus),
+            "count_order": r.count_order, "sum_qty": r.sum_qty, "sum_base_price": r.sum_base_price,
+            "sum_disc_price": (r.sum_disc_price_hi << 64) | r.sum_disc_price_lo,
+            "sum_charge": (r.sum_charge_hi << 64) | r.sum_charge_lo, "sum_disc": r.sum_disc,
+            "avg_qty": r.avg_qty, "avg_price": r.avg_price, "avg_disc": r.avg_disc,
+        })
+    return out, rc
+
+
+def fission_run(h_in, preds, chunk_rows: int, streams, fused: bool = True, h_out=None,
+                h_chunk_counts=None, device=None):
+    """Host-resident SELECT chain with kernel fission (synchronous).
+
+    ``h_in``: pinned CPU int32 tensor.  Returns ``(h_out, count)`` with
+    ``h_out[:count]`` the selected values.
+    """
+    torch = _torch()
+    if not (h_in.dtype == torch.int32 and h_in.is_contiguous() and (h_in.numel() == 0 or h_in.is_pinned())):
+        raise ValueError("h_in must be a pinned contiguous int32 CPU tensor")
+    n, k = h_in.numel(), len(preds)
+    chunk_rows = max(1, min(int(chunk_rows), max(1, n)))
+    nchunks = (n + chunk_rows - 1) // chunk_rows
+    device = device or torch.device("cuda", torch.cuda.current_device())
+    if h_out is None:
+        h_out = torch.empty(max(1, n), dtype=torch.int32, pin_memory=True)
+    if h_chunk_counts is None or h_chunk_counts.numel() < max(1, nchunks):
+        h_chunk_counts = torch.zeros(max(1, nchunks), dtype=torch.int64, pin_memory=True)
+    S = len(streams)
+    sarr = (ctypes.c_void_p * S)(*[_stream_handle(s) for s in streams])
+    ws = workspace(device, f"fission_{int(fused)}_{S}", ra_fission_workspace_bytes(chunk_rows, S, k, int(fused)))
+    P = make_preds(preds)
+    cnt = ctypes.c_int64(0)
+    ra_fission_run(h_in.data_ptr(), n, P, k, int(fused), chunk_rows, sarr, S, h_out.data_ptr(),
+                   h_out.numel(), ctypes.byref(cnt), h_chunk_counts.data_ptr(), ws.data_ptr(),
+                   ws.numel())
+    return h_out, int(cnt.value)

@@ -1,0 +1,244 @@
+// capi.cu — extern "C" entry points of libra.so (declared in include/ra.h):
+// argument validation, workspace sizing, dispatch to the kernels, and the
+// host-side Q1 finalize.  No allocation, no exceptions across the ABI.
+
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include "ra_internal.cuh"
+
+namespace ra {
+
+std::atomic<uint64_t> g_launches{0};
+
+namespace {
+thread_local char t_err[512] = "";
+}
+
+void clear_error() { t_err[0] = 0; }
+
+int fail(int code, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(t_err, sizeof(t_err), fmt, ap);
+  va_end(ap);
+  return code;
+}
+
+int cuda_fail(cudaError_t e, const char* what) {
+  return fail(RA_E_CUDA, "%s: %s (%d)", what, cudaGetErrorString(e), (int)e);
+}
+
+int num_sms() {
+  static int cache[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
+  if (!cache[dev]) {
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    cache[dev] = v > 0 ? v : 148;
+  }
+  return cache[dev];
+}
+
+int canonicalize(const ra_pred* preds, int k, CanonPred* out) {
+  int32_t lo = INT32_MIN, hi = INT32_MAX;
+  bool empty = false;
+  int n_ne = 0;
+  int32_t ne[RA_MAX_PREDS];
+  for (int j = 0; j < k; ++j) {
+    const int32_t v = preds[j].value;
+    switch (preds[j].op) {
+      case RA_LT:
+        if (v == INT32_MIN) empty = true;
+        else if (v - 1 < hi) hi = v - 1;
+        break;
+      case RA_LE:
+        if (v < hi) hi = v;
+        break;
+      case RA_GT:
+        if (v == INT32_MAX) empty = true;
+        else if (v + 1 > lo) lo = v + 1;
+        break;
+      case RA_GE:
+        if (v > lo) lo = v;
+        break;
+      case RA_EQ:
+        if (v > lo) lo = v;
+        if (v < hi) hi = v;
+        break;
+      case RA_NE: {
+        bool dup = false;
+        for (int i = 0; i < n_ne; ++i) dup |= (ne[i] == v);
+        if (!dup) ne[n_ne++] = v;
+        break;
+      }
+      default:
+        return fail(RA_E_INVAL, "predicate %d: unknown op %d", j, (int)preds[j].op);
+    }
+  }
+  if (empty || lo > hi) {
+    lo = 1;
+    hi = 0;  // empty interval
+    n_ne = 0;
+  }
+  // drop exclusions outside the interval; an exclusion at an end shrinks it
+  bool changed = true;
+  while (changed && lo <= hi) {
+    changed = false;
+    for (int i = 0; i < n_ne; ++i) {
+      if (ne[i] < lo || ne[i] > hi) {
+        ne[i--] = ne[--n_ne];
+        changed = true;
+      } else if (ne[i] == lo && lo < hi) {
+        lo = lo + 1;
+        ne[i--] = ne[--n_ne];
+        changed = true;
+      } else if (ne[i] == hi && lo < hi) {
+        hi = hi - 1;
+        ne[i--] = ne[--n_ne];
+        changed = true;
+      } else if (lo == hi && ne[i] == lo) {
+        lo = 1;
+        hi = 0;
+        n_ne = 0;
+        changed = false;
+        break;
+      }
+    }
+  }
+  out->lo = lo;
+  out->hi = hi;
+  out->n_ne = n_ne;
+  for (int i = 0; i < RA_MAX_PREDS; ++i) out->ne[i] = i < n_ne ? ne[i] : 0;
+  return RA_OK;
+}
+
+}  // namespace ra
+
+using namespace ra;
+
+RA_API const char* ra_last_error(void) { return t_err; }
+RA_API int ra_version(void) { return 1; }
+RA_API uint64_t ra_kernel_launches(void) { return g_launches.load(std::memory_order_relaxed); }
+
+RA_API int ra_workspace_init(void* d_ws, size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  if (ws_bytes == 0) return RA_OK;
+  if (!d_ws) return fail(RA_E_INVAL, "null workspace");
+  cudaError_t e = cudaMemsetAsync(d_ws, 0, ws_bytes, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(workspace)");
+  return RA_OK;
+}
+
+RA_API size_t ra_select_workspace_bytes(int64_t n, int k, int fused) {
+  if (n < 0) n = 0;
+  size_t b = (sel_status_bytes(n) + 255) / 256 * 256;
+  if (!fused && k > 1) b += sel_inter_bytes(n);
+  return b;
+}
+
+static int check_select_args(const int32_t* d_in, int64_t n, int k, int32_t* d_out, int64_t out_cap,
+                             int64_t* d_count, void* d_ws, size_t ws_bytes, int fused) {
+  if (n < 0 || out_cap < 0) return fail(RA_E_INVAL, "negative n or out_cap");
+  if (k < 0 || k > RA_MAX_PREDS) return fail(RA_E_INVAL, "k=%d outside [0, %d]", k, RA_MAX_PREDS);
+  if (!d_count || !d_ws) return fail(RA_E_INVAL, "null d_count or workspace");
+  if (n > 0 && !d_in) return fail(RA_E_INVAL, "null d_in with n > 0");
+  if (out_cap > 0 && !d_out) return fail(RA_E_INVAL, "null d_out with out_cap > 0");
+  if (((uintptr_t)d_in | (uintptr_t)d_out) & 3u) return fail(RA_E_INVAL, "pointers must be 4-byte aligned");
+  if ((uintptr_t)d_count & 7u) return fail(RA_E_INVAL, "d_count must be 8-byte aligned");
+  if ((uintptr_t)d_ws & 255u) return fail(RA_E_INVAL, "workspace must be 256-byte aligned");
+  const size_t need = ra_select_workspace_bytes(n, k, fused);
+  if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
+  return RA_OK;
+}
+
+RA_API int ra_select(const int32_t* d_in, int64_t n, ra_pred pred, int32_t* d_out, int64_t out_cap,
+                     int64_t* d_count, void* d_ws, size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  int rc = check_select_args(d_in, n, 1, d_out, out_cap, d_count, d_ws, ws_bytes, 1);
+  if (rc) return rc;
+  return select_chain_impl(d_in, n, &pred, 1, 1, d_out, out_cap, d_count, d_ws, ws_bytes,
+                           (cudaStream_t)stream);
+}
+
+RA_API int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,
+                           int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                           size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  int rc = check_select_args(d_in, n, k, d_out, out_cap, d_count, d_ws, ws_bytes, fused);
+  if (rc) return rc;
+  if (k > 0 && !h_preds) return fail(RA_E_INVAL, "null h_preds with k > 0");
+  for (int j = 0; j < k; ++j)
+    if (h_preds[j].op < RA_LT || h_preds[j].op > RA_NE)
+      return fail(RA_E_INVAL, "predicate %d: unknown op %d", j, (int)h_preds[j].op);
+  return select_chain_impl(d_in, n, h_preds, k, fused, d_out, out_cap, d_count, d_ws, ws_bytes,
+                           (cudaStream_t)stream);
+}
+
+RA_API size_t ra_q1_workspace_bytes(int64_t n) {
+  (void)n;
+  return q1_ws_bytes();
+}
+
+RA_API int ra_q1(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff, ra_q1_partial* d_partial,
+                 void* d_ws, size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  if (!h_cols || !d_partial || !d_ws) return fail(RA_E_INVAL, "null argument");
+  if (n < 0 || n >= (int64_t)1 << 32) return fail(RA_E_INVAL, "n=%lld outside [0, 2^32)", (long long)n);
+  const ra_lineitem& c = *h_cols;
+  if (n > 0 && (!c.shipdate || !c.returnflag || !c.linestatus || !c.quantity || !c.extendedprice ||
+                !c.discount || !c.tax))
+    return fail(RA_E_INVAL, "null column with n > 0");
+  if (((uintptr_t)c.shipdate & 3u) || (((uintptr_t)c.quantity | (uintptr_t)c.extendedprice |
+                                        (uintptr_t)c.discount | (uintptr_t)c.tax) & 7u))
+    return fail(RA_E_INVAL, "columns must be naturally aligned");
+  if ((uintptr_t)d_partial & 7u) return fail(RA_E_INVAL, "d_partial must be 8-byte aligned");
+  if ((uintptr_t)d_ws & 255u) return fail(RA_E_INVAL, "workspace must be 256-byte aligned");
+  if (ws_bytes < q1_ws_bytes()) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, q1_ws_bytes());
+  return launch_q1(c, n, shipdate_cutoff, d_partial, d_ws, ws_bytes, (cudaStream_t)stream);
+}
+
+RA_API int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h_rows, int* n_rows) {
+  clear_error();
+  if (n_partials < 0 || (n_partials > 0 && !h_partials) || !h_rows || !n_rows)
+    return fail(RA_E_INVAL, "null argument");
+  static const uint8_t RF[3] = {'A', 'N', 'R'}, LS[2] = {'F', 'O'};
+  uint32_t status = 0;
+  int m = 0;
+  for (int s = 0; s < RA_Q1_GROUPS; ++s) {  // slot order == ORDER BY (rf, ls)
+    int64_t cnt = 0, sq = 0, sp = 0, sd = 0;
+    unsigned __int128 dp = 0, ch = 0;
+    for (int i = 0; i < n_partials; ++i) {
+      const ra_q1_group& g = h_partials[i].group[s];
+      if (s == 0) status |= h_partials[i].status;
+      cnt += g.count;
+      sq += g.sum_qty;
+      sp += g.sum_base_price;
+      sd += g.sum_disc;
+      dp += ((unsigned __int128)(uint64_t)g.sum_disc_price_hi << 64) | g.sum_disc_price_lo;
+      ch += ((unsigned __int128)(uint64_t)g.sum_charge_hi << 64) | g.sum_charge_lo;
+    }
+    if (cnt == 0) continue;  // GROUP BY emits no empty groups
+    ra_q1_row& r = h_rows[m++];
+    memset(&r, 0, sizeof(r));
+    r.returnflag = RF[s >> 1];
+    r.linestatus = LS[s & 1];
+    r.count_order = cnt;
+    r.sum_qty = sq;
+    r.sum_base_price = sp;
+    r.sum_disc = sd;
+    r.sum_disc_price_lo = (uint64_t)dp;
+    r.sum_disc_price_hi = (int64_t)(uint64_t)(dp >> 64);
+    r.sum_charge_lo = (uint64_t)ch;
+    r.sum_charge_hi = (int64_t)(uint64_t)(ch >> 64);
+    const double den = (double)(cnt * 100);  // one division of exact operands (C12)
+    r.avg_qty = (double)sq / den;
+    r.avg_price = (double)sp / den;
+    r.avg_disc = (double)sd / den;
+  }
+  *n_rows = m;
+  if (status) return fail(RA_E_DOMAIN, "Q1 input outside the domain (status 0x%x)", status);
+  return RA_OK;
+}

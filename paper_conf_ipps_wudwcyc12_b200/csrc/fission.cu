@@ -1,0 +1,170 @@
+// fission.cu — kernel fission for a host-resident SELECT chain (§IV).
+//
+// The paper's Stream Pool (Table IV) hands out CUDA
+// streams and per-stream command lists; fission partitions a kernel into
+// segments whose PCIe transfers overlap the computation of other segments
+// (Fig 13), and a fused kernel under fission needs a CPU gather
+// because "data is transferred to the CPU at different times" (§IV-C,
+// L1456-1468).  This runner is that pool specialised to one pipeline:
+//
+//   chunk c -> stream c mod S:  H2D(chunk c)  ->  select_fused(chunk c)
+//           -> count written straight into pinned h_chunk_counts[c] (mapped)
+//   host, once chunk c's kernel event fires: D2H of exactly count_c values
+//           into h_out + running offset  (the CPU gather as placement)
+//
+// The host waits on chunk c only when it is about to reuse chunk c's stream
+// buffers (S chunks later), so S-1 H2D copies stay queued ahead of it and the
+// copy engines never idle on a host round trip.
+
+#include <stdio.h>
+#include <string.h>
+
+#include <vector>
+
+#include "ra_internal.cuh"
+
+namespace ra {
+
+namespace {
+
+size_t round256(size_t b) { return (b + 255) / 256 * 256; }
+
+size_t per_stream_bytes(int64_t chunk_rows, int k, int fused) {
+  const size_t io = round256((size_t)chunk_rows * 4);
+  return 2 * io + round256(ra_select_workspace_bytes(chunk_rows, k, fused));
+}
+
+int check_pinned(const void* p, const char* name, void** dev_alias) {
+  cudaPointerAttributes a;
+  cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(RA_E_NOT_PINNED, "%s: not a CUDA-registered host pointer", name);
+  }
+  if (a.type != cudaMemoryTypeHost) return fail(RA_E_NOT_PINNED, "%s is not page-locked host memory", name);
+  if (dev_alias) {
+    *dev_alias = a.devicePointer;
+    if (!*dev_alias) return fail(RA_E_NOT_PINNED, "%s has no device mapping", name);
+  }
+  return RA_OK;
+}
+
+}  // namespace
+
+}  // namespace ra
+
+using namespace ra;
+
+RA_API size_t ra_fission_workspace_bytes(int64_t chunk_rows, int n_streams, int k, int fused) {
+  if (chunk_rows <= 0 || n_streams <= 0) return 0;
+  return (size_t)n_streams * per_stream_bytes(chunk_rows, k, fused);
+}
+
+RA_API int ra_fission_run(const int32_t* h_in, int64_t n, const ra_pred* h_preds, int k, int fused,
+                          int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
+                          int32_t* h_out, int64_t out_cap, int64_t* h_count,
+                          int64_t* h_chunk_counts, void* d_ws, size_t ws_bytes) {
+  clear_error();
+  if (n < 0 || k < 0 || k > RA_MAX_PREDS || chunk_rows <= 0 || n_streams <= 0 || out_cap < 0)
+    return fail(RA_E_INVAL, "bad sizes (n=%lld k=%d chunk_rows=%lld n_streams=%d)", (long long)n, k,
+                (long long)chunk_rows, n_streams);
+  if (!h_count || !streams || (k > 0 && !h_preds)) return fail(RA_E_INVAL, "null argument");
+  if (n > 0 && (!h_in || !h_chunk_counts || !d_ws || (out_cap > 0 && !h_out)))
+    return fail(RA_E_INVAL, "null buffer with n > 0");
+  if (((uintptr_t)h_in | (uintptr_t)h_out) & 3u) return fail(RA_E_INVAL, "host buffers must be 4-byte aligned");
+  CanonPred cp;
+  for (int j = 0; j < k; ++j) {
+    int rc = canonicalize(&h_preds[j], 1, &cp);
+    if (rc) return rc;
+  }
+  if (n == 0) {
+    *h_count = 0;
+    return RA_OK;
+  }
+  if (chunk_rows > n) chunk_rows = n;
+  const size_t need = ra_fission_workspace_bytes(chunk_rows, n_streams, k, fused);
+  if (ws_bytes < need)
+    return fail(RA_E_WORKSPACE, "fission workspace %zu < required %zu", ws_bytes, need);
+  int rc = check_pinned(h_in, "h_in", nullptr);
+  if (rc) return rc;
+  if (out_cap > 0 && (rc = check_pinned(h_out, "h_out", nullptr))) return rc;
+  void* counts_alias = nullptr;
+  if ((rc = check_pinned(h_chunk_counts, "h_chunk_counts", &counts_alias))) return rc;
+  int64_t* d_counts = (int64_t*)counts_alias;
+
+  const int S = n_streams;
+  const size_t per = per_stream_bytes(chunk_rows, k, fused);
+  const size_t io = round256((size_t)chunk_rows * 4);
+  std::vector<cudaEvent_t> ev(S);
+  for (int s = 0; s < S; ++s) {
+    cudaError_t e = cudaEventCreateWithFlags(&ev[s], cudaEventDisableTiming);
+    if (e != cudaSuccess) {
+      for (int j = 0; j < s; ++j) cudaEventDestroy(ev[j]);
+      return cuda_fail(e, "cudaEventCreate");
+    }
+  }
+  // The per-stream select workspaces move with chunk_rows: re-zero their
+  // control words (header + status, a few KB) so earlier calls' data in this
+  // workspace can never read as tile status.
+  for (int s = 0; s < S; ++s) {
+    char* base = (char*)d_ws + (size_t)s * per;
+    cudaError_t e = cudaMemsetAsync(base + 2 * io, 0, sel_status_bytes(chunk_rows), (cudaStream_t)streams[s]);
+    if (e != cudaSuccess) {
+      for (int j = 0; j < S; ++j) cudaEventDestroy(ev[j]);
+      return cuda_fail(e, "cudaMemsetAsync(fission control words)");
+    }
+  }
+  const int64_t C = (n + chunk_rows - 1) / chunk_rows;
+  int64_t offset = 0;  // running output offset (CPU gather)
+  int result = RA_OK;
+
+  auto gather = [&](int64_t c) -> int {
+    const int s = (int)(c % S);
+    cudaError_t e = cudaEventSynchronize(ev[s]);
+    if (e != cudaSuccess) return cuda_fail(e, "chunk event");
+    const int64_t cnt = ((volatile int64_t*)h_chunk_counts)[c];
+    int64_t ncopy = out_cap - offset;
+    ncopy = ncopy < 0 ? 0 : (ncopy > cnt ? cnt : ncopy);
+    if (ncopy > 0) {
+      char* base = (char*)d_ws + (size_t)s * per;
+      e = cudaMemcpyAsync(h_out + offset, base + io, (size_t)ncopy * 4, cudaMemcpyDeviceToHost,
+                          (cudaStream_t)streams[s]);
+      if (e != cudaSuccess) return cuda_fail(e, "D2H chunk result");
+    }
+    offset += cnt;
+    return RA_OK;
+  };
+
+  for (int64_t c = 0; c < C && result == RA_OK; ++c) {
+    const int s = (int)(c % S);
+    if (c >= S && (result = gather(c - S)) != RA_OK) break;
+    const int64_t r0 = c * chunk_rows;
+    const int64_t len = (n - r0 < chunk_rows) ? (n - r0) : chunk_rows;
+    char* base = (char*)d_ws + (size_t)s * per;
+    int32_t* d_in = (int32_t*)base;
+    int32_t* d_out = (int32_t*)(base + io);
+    void* sel_ws = base + 2 * io;
+    cudaStream_t st = (cudaStream_t)streams[s];
+    cudaError_t e = cudaMemcpyAsync(d_in, h_in + r0, (size_t)len * 4, cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) {
+      result = cuda_fail(e, "H2D chunk");
+      break;
+    }
+    result = select_chain_impl(d_in, len, h_preds, k, fused, d_out, len, d_counts + c, sel_ws,
+                               per - 2 * io, st);
+    if (result != RA_OK) break;
+    e = cudaEventRecord(ev[s], st);
+    if (e != cudaSuccess) result = cuda_fail(e, "cudaEventRecord");
+  }
+  for (int64_t c = (C > S ? C - S : 0); c < C && result == RA_OK; ++c) result = gather(c);
+  for (int s = 0; s < S; ++s) {
+    cudaError_t e = cudaStreamSynchronize((cudaStream_t)streams[s]);
+    if (e != cudaSuccess && result == RA_OK) result = cuda_fail(e, "stream sync");
+    cudaEventDestroy(ev[s]);
+  }
+  if (result != RA_OK) return result;
+  *h_count = offset;
+  if (offset > out_cap)
+    return fail(RA_E_CAPACITY, "%lld selected > out_cap %lld", (long long)offset, (long long)out_cap);
+  return RA_OK;
+}

@@ -1,0 +1,340 @@
+// q1_fused.cu — TPC-H Q1 as one fused kernel for sm_100a.
+//
+// The paper's Q1 plan (Fig 17(a), §V) is SELECT + six
+// JOINs (fused) -> SORT by (returnflag, linestatus) -> fused arithmetic ->
+// aggregate/unique; SORT alone was ~71% of the baseline (L1576-1577) and the
+// fusible part gained 3.18x (L1673-1676).  In a positional column store the
+// JOINs are identities and the SORT only orders <= 6 groups, so
+// the whole query becomes one streaming pass:
+//
+//   SELECT   shipdate <= cutoff                              (Fig 2(g))
+//   PROJECT  disc_price = price*(100-disc), charge = disc_price*(100+tax)
+//            computed in registers, never stored             (Fig 2(h))
+//   GROUP BY slot = 2*rf + ls into per-thread register accumulators (6 slots),
+//            reduced warp -> CTA -> grid at the end; the last CTA to finish
+//            folds the CTA partials (threadfence + ticket) in 128-bit.
+//
+// Loads: 4 rows per thread per step as one int4 (shipdate), two u32 (flags)
+// and two int4 per decimal column — all coalesced 128-bit except the flag
+// words; two steps are issued back to back for memory-level parallelism.
+// Persistent grid (SM count x occupancy), grid-stride over 4-row groups.
+//
+// Exactness: in the documented domain (ra.h) a row's
+// disc_price < 2^38 and charge < 2^46.  Each thread handles <= 2^17 rows
+// (enforced by the grid size for n < 2^32) so its 64-bit sums cannot wrap;
+// warp, CTA and grid sums of disc_price and charge are 128-bit.
+
+#include <stdio.h>
+
+#include "ra_internal.cuh"
+
+namespace ra {
+
+namespace {
+
+constexpr int Q1_THREADS = 256;
+constexpr int Q1_MAX_GRID = 148 * 8;
+constexpr int NS = RA_Q1_GROUPS;
+
+struct Q1Block {
+  uint32_t status;
+  uint32_t _pad;
+  uint64_t v[NS][8];  // count, qty, price, disc, dp_lo, dp_hi, ch_lo, ch_hi
+};
+
+struct Q1Params {
+  const int32_t* sd;
+  const uint8_t* rf;
+  const uint8_t* ls;
+  const int64_t* q;
+  const int64_t* p;
+  const int64_t* d;
+  const int64_t* t;
+  int64_t n;
+  int64_t head;     // rows before the first 4-row aligned group
+  int64_t ngroups;  // aligned 4-row groups starting at `head`
+  int32_t cutoff;
+  ra_q1_partial* out;
+  Q1Block* blocks;
+  uint32_t* counter;
+};
+
+struct Acc {
+  uint32_t cnt[NS];
+  uint32_t sdisc[NS];
+  uint64_t sq[NS], sp[NS], sdp[NS], sch[NS];
+  uint32_t status;
+};
+
+__device__ __forceinline__ void row(Acc& A, int32_t cutoff, int32_t sd, uint32_t rfb, uint32_t lsb,
+                                    int64_t q, int64_t p, int64_t d, int64_t t) {
+  const bool sel = sd <= cutoff;  // SELECT
+  const int ri = rfb == 'A' ? 0 : rfb == 'N' ? 2 : rfb == 'R' ? 4 : -8;
+  const int li = lsb == 'F' ? 0 : lsb == 'O' ? 1 : -8;
+  const bool okf = (ri | li) >= 0;
+  const bool okn = ((uint64_t)q < (1ull << 31)) & ((uint64_t)p < (1ull << 31)) &
+                   ((uint64_t)d <= 100ull) & ((uint64_t)t <= 100ull);
+  A.status |= sel ? ((okf ? 0u : 1u) | (okn ? 0u : 2u)) : 0u;
+  const int slot = (sel & okf & okn) ? (ri + li) : -1;
+  // PROJECT (exact in the domain: 32x32->64 and 64x32 products)
+  const uint64_t dp = (uint64_t)(uint32_t)p * (uint32_t)(100 - (uint32_t)d);
+  const uint64_t ch = dp * (uint64_t)(100u + (uint32_t)t);
+  // GROUP BY into register slots (predicated adds)
+#pragma unroll
+  for (int s = 0; s < NS; ++s) {
+    if (slot == s) {
+      A.cnt[s] += 1;
+      A.sq[s] += (uint64_t)q;
+      A.sp[s] += (uint64_t)p;
+      A.sdp[s] += dp;
+      A.sch[s] += ch;
+      A.sdisc[s] += (uint32_t)d;
+    }
+  }
+}
+
+struct Group4 {
+  int4 sd;
+  uint32_t rf, ls;
+  longlong2 q[2], p[2], d[2], t[2];
+};
+
+__device__ __forceinline__ longlong2 ld_stream_ll2(const int64_t* ptr) {
+  longlong2 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v2.s64 {%0,%1}, [%2];" : "=l"(r.x), "=l"(r.y) : "l"(ptr));
+  return r;
+}
+
+__device__ __forceinline__ uint32_t ld_stream_u32(const uint8_t* ptr) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(ptr));
+  return r;
+}
+
+__device__ __forceinline__ void load_group(Group4& G, const Q1Params& P, int64_t g) {
+  const int64_t r = P.head + 4 * g;
+  G.sd = dev::ld_stream_v4((const int4*)(P.sd + r));
+  G.rf = ld_stream_u32(P.rf + r);
+  G.ls = ld_stream_u32(P.ls + r);
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    G.q[h] = ld_stream_ll2(P.q + r + 2 * h);
+    G.p[h] = ld_stream_ll2(P.p + r + 2 * h);
+    G.d[h] = ld_stream_ll2(P.d + r + 2 * h);
+    G.t[h] = ld_stream_ll2(P.t + r + 2 * h);
+  }
+}
+
+__device__ __forceinline__ void process_group(Acc& A, const Group4& G, int32_t cutoff) {
+  row(A, cutoff, G.sd.x, G.rf & 0xFF, G.ls & 0xFF, G.q[0].x, G.p[0].x, G.d[0].x, G.t[0].x);
+  row(A, cutoff, G.sd.y, (G.rf >> 8) & 0xFF, (G.ls >> 8) & 0xFF, G.q[0].y, G.p[0].y, G.d[0].y, G.t[0].y);
+  row(A, cutoff, G.sd.z, (G.rf >> 16) & 0xFF, (G.ls >> 16) & 0xFF, G.q[1].x, G.p[1].x, G.d[1].x, G.t[1].x);
+  row(A, cutoff, G.sd.w, G.rf >> 24, G.ls >> 24, G.q[1].y, G.p[1].y, G.d[1].y, G.t[1].y);
+}
+
+__device__ __forceinline__ void add128(uint64_t& lo, uint64_t& hi, uint64_t lo2, uint64_t hi2) {
+  const uint64_t l = lo + lo2;
+  hi += hi2 + (l < lo ? 1ull : 0ull);
+  lo = l;
+}
+
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+__device__ __forceinline__ void warp_sum_u128(uint64_t& lo, uint64_t& hi) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const uint64_t l2 = __shfl_xor_sync(0xffffffffu, lo, o);
+    const uint64_t h2 = __shfl_xor_sync(0xffffffffu, hi, o);
+    add128(lo, hi, l2, h2);
+  }
+}
+
+__global__ void __launch_bounds__(Q1_THREADS, 2) q1_fused_kernel(const Q1Params P) {
+  __shared__ uint64_t s_w[Q1_THREADS / 32][NS][8];
+  __shared__ uint32_t s_status;
+  __shared__ bool s_last;
+
+  Acc A;
+#pragma unroll
+  for (int s = 0; s < NS; ++s) {
+    A.cnt[s] = 0;
+    A.sdisc[s] = 0;
+    A.sq[s] = A.sp[s] = A.sdp[s] = A.sch[s] = 0;
+  }
+  A.status = 0;
+  if (threadIdx.x == 0) s_status = 0;
+
+  const int64_t gtid = (int64_t)blockIdx.x * Q1_THREADS + threadIdx.x;
+  const int64_t gstride = (int64_t)gridDim.x * Q1_THREADS;
+
+  // aligned 4-row groups (10 x 128-bit loads in flight per thread per group)
+  for (int64_t g = gtid; g < P.ngroups; g += gstride) {
+    Group4 G0;
+    load_group(G0, P, g);
+    process_group(A, G0, P.cutoff);
+  }
+  // scalar rows: [0, head) and the tail after the aligned groups
+  const int64_t tail0 = P.head + 4 * P.ngroups;
+  const int64_t nscalar = P.head + (P.n - tail0);
+  for (int64_t i = gtid; i < nscalar; i += gstride) {
+    const int64_t r = i < P.head ? i : tail0 + (i - P.head);
+    row(A, P.cutoff, P.sd[r], P.rf[r], P.ls[r], P.q[r], P.p[r], P.d[r], P.t[r]);
+  }
+
+  // ---- reduction: warp (shuffles) -> CTA (smem) -> grid (last CTA)
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (A.status) atomicOr(&s_status, A.status);
+#pragma unroll
+  for (int s = 0; s < NS; ++s) {
+    const uint64_t c = warp_sum_u64(A.cnt[s]);
+    const uint64_t q = warp_sum_u64(A.sq[s]);
+    const uint64_t p = warp_sum_u64(A.sp[s]);
+    const uint64_t d = warp_sum_u64(A.sdisc[s]);
+    uint64_t dlo = A.sdp[s], dhi = 0, clo = A.sch[s], chi = 0;
+    warp_sum_u128(dlo, dhi);
+    warp_sum_u128(clo, chi);
+    if (lane == 0) {
+      s_w[warp][s][0] = c;
+      s_w[warp][s][1] = q;
+      s_w[warp][s][2] = p;
+      s_w[warp][s][3] = d;
+      s_w[warp][s][4] = dlo;
+      s_w[warp][s][5] = dhi;
+      s_w[warp][s][6] = clo;
+      s_w[warp][s][7] = chi;
+    }
+  }
+  __syncthreads();
+  Q1Block* mine = P.blocks + blockIdx.x;
+  if (threadIdx.x < NS * 4) {  // (slot, field pair)
+    const int s = threadIdx.x >> 2, f = threadIdx.x & 3;
+    if (f < 2) {  // count/qty or price/disc: 64-bit
+      uint64_t a = 0, b = 0;
+      for (int w = 0; w < Q1_THREADS / 32; ++w) {
+        a += s_w[w][s][2 * f];
+        b += s_w[w][s][2 * f + 1];
+      }
+      mine->v[s][2 * f] = a;
+      mine->v[s][2 * f + 1] = b;
+    } else {  // dp or ch: 128-bit
+      uint64_t lo = 0, hi = 0;
+      for (int w = 0; w < Q1_THREADS / 32; ++w) add128(lo, hi, s_w[w][s][2 * f], s_w[w][s][2 * f + 1]);
+      mine->v[s][2 * f] = lo;
+      mine->v[s][2 * f + 1] = hi;
+    }
+  }
+  if (threadIdx.x == 0) mine->status = s_status;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = (atomicAdd(P.counter, 1u) == gridDim.x - 1);
+  __syncthreads();
+  if (!s_last) return;
+
+  // ---- last CTA: fold all CTA partials (128-bit where needed)
+  __threadfence();
+  const int nb = gridDim.x;
+  if (threadIdx.x < NS * 4) {
+    const int s = threadIdx.x >> 2, f = threadIdx.x & 3;
+    uint64_t a = 0, b = 0;
+    for (int i = 0; i < nb; ++i) {
+      const uint64_t x = __ldcg(&P.blocks[i].v[s][2 * f]);
+      const uint64_t y = __ldcg(&P.blocks[i].v[s][2 * f + 1]);
+      if (f < 2) {
+        a += x;
+        b += y;
+      } else {
+        add128(a, b, x, y);
+      }
+    }
+    ra_q1_group* G = &P.out->group[s];
+    if (f == 0) {
+      G->count = (int64_t)a;
+      G->sum_qty = (int64_t)b;
+    } else if (f == 1) {
+      G->sum_base_price = (int64_t)a;
+      G->sum_disc = (int64_t)b;
+    } else if (f == 2) {
+      G->sum_disc_price_lo = a;
+      G->sum_disc_price_hi = (int64_t)b;
+    } else {
+      G->sum_charge_lo = a;
+      G->sum_charge_hi = (int64_t)b;
+    }
+  } else if (threadIdx.x == 32) {
+    uint32_t st = 0;
+    for (int i = 0; i < nb; ++i) st |= __ldcg(&P.blocks[i].status);
+    P.out->status = st;
+    P.out->n_groups = NS;
+    P.out->rows = (uint64_t)P.n;
+    *P.counter = 0u;  // self-cleaning for the next launch
+  }
+}
+
+int g_q1_occ[64];  // blocks/SM per device (0 = unknown)
+
+}  // namespace
+
+size_t q1_ws_bytes() { return 256 + (size_t)Q1_MAX_GRID * sizeof(Q1Block); }
+
+int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_partial, void* d_ws,
+              size_t ws_bytes, cudaStream_t s) {
+  (void)ws_bytes;
+  Q1Params P;
+  P.sd = c.shipdate;
+  P.rf = c.returnflag;
+  P.ls = c.linestatus;
+  P.q = c.quantity;
+  P.p = c.extendedprice;
+  P.d = c.discount;
+  P.t = c.tax;
+  P.n = n;
+  P.cutoff = cutoff;
+  P.out = d_partial;
+  P.counter = (uint32_t*)d_ws;
+  P.blocks = (Q1Block*)((char*)d_ws + 256);
+  // first row index h at which every column is 16-B (flags: 4-B) aligned
+  P.head = n;
+  P.ngroups = 0;
+  for (int64_t h = 0; h < 16 && h < n; ++h) {
+    const bool ok = ((uintptr_t)(c.shipdate + h) % 16 == 0) && ((uintptr_t)(c.returnflag + h) % 4 == 0) &&
+                    ((uintptr_t)(c.linestatus + h) % 4 == 0) && ((uintptr_t)(c.quantity + h) % 16 == 0) &&
+                    ((uintptr_t)(c.extendedprice + h) % 16 == 0) && ((uintptr_t)(c.discount + h) % 16 == 0) &&
+                    ((uintptr_t)(c.tax + h) % 16 == 0);
+    if (ok) {
+      P.head = h;
+      P.ngroups = (n - h) / 4;
+      break;
+    }
+  }
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (g_q1_occ[dev] == 0) {
+    int occ = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, q1_fused_kernel, Q1_THREADS, 0);
+    if (e != cudaSuccess) return cuda_fail(e, "occupancy query");
+    g_q1_occ[dev] = occ > 0 ? occ : 1;
+  }
+  int64_t grid = (int64_t)num_sms() * g_q1_occ[dev];
+  if (grid > Q1_MAX_GRID) grid = Q1_MAX_GRID;
+  const int64_t work = P.ngroups > 0 ? P.ngroups : n;
+  const int64_t need = (work + Q1_THREADS - 1) / Q1_THREADS;
+  if (grid > need) grid = need;
+  // per-thread 64-bit sums stay exact while rows/thread <= 2^17
+  const int64_t min_grid = (n >> 17) / Q1_THREADS + 1;
+  if (grid < min_grid) grid = min_grid;
+  if (grid < 1) grid = 1;
+  if (grid > Q1_MAX_GRID) return fail(RA_E_INVAL, "n too large for the Q1 grid");
+  q1_fused_kernel<<<(unsigned)grid, Q1_THREADS, 0, s>>>(P);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "q1_fused_kernel launch");
+  return RA_OK;
+}
+
+}  // namespace ra

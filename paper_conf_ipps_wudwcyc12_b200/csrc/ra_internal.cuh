@@ -1,0 +1,128 @@
+// ra_internal.cuh — shared internals of libra.so (product side only; the
+// oracle shares none of this).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "ra.h"
+
+#define RA_API extern "C" __attribute__((visibility("default")))
+
+namespace ra {
+
+// ------------------------------------------------------------ errors
+int fail(int code, const char* fmt, ...);  // sets the thread-local message, returns code
+int cuda_fail(cudaError_t e, const char* what);
+void clear_error();
+
+extern std::atomic<uint64_t> g_launches;
+inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+int num_sms();  // of the current device (cached per device)
+
+// ------------------------------------------------- predicate canonical form
+// A conjunction of k (op, value) predicates on a signed int32 equals
+//   lo <= x <= hi  and  x != ne[0..n_ne)
+// (an empty interval when lo > hi).  Folding the chain once on the host is the
+// Table III observation: the fused "d<T1 && d<T2" compiles
+// to the instructions of a single compare.
+struct CanonPred {
+  int32_t lo, hi;
+  int32_t n_ne;
+  int32_t ne[RA_MAX_PREDS];
+};
+int canonicalize(const ra_pred* preds, int k, CanonPred* out);
+
+// ------------------------------------------------------------ SELECT
+constexpr int SEL_THREADS = 256;  // compute threads per CTA (plus one look-back warp)
+constexpr int SEL_VEC = 4;        // int4 vectors per compute thread per tile
+constexpr int SEL_AHEAD = 2;      // tiles whose bulk copy is in flight ahead of the count
+constexpr int SEL_INSLOTS = SEL_AHEAD + 1;           // input ring slots (tiles)
+constexpr int SEL_LAG = 5;        // a tile is written SEL_LAG tiles after it is counted (or earlier)
+constexpr int SEL_OUTRING = 13312;                   // compacted-row ring (int32), 52 KB
+constexpr int SEL_TILE = SEL_THREADS * SEL_VEC * 4;  // 4096 rows / tile
+int sel_ctas_per_sm();  // occupancy of the select kernel on the current device
+
+// Workspace layout (see select_fused.cu):
+//   [0, 256)                       header (launch epoch)
+//   [256, 256 + 8 * ntiles)        status words (epoch-tagged)
+//   [W - inter, W)                 unfused only: two int32[n] + 2 int64 counts
+constexpr size_t SEL_HDR_BYTES = 256;
+int64_t sel_max_tiles(int64_t n);  // tiles for n rows with any 16-B misalignment
+size_t sel_status_bytes(int64_t n);
+size_t sel_inter_bytes(int64_t n);
+
+// One select pass (one kernel).  n_max = host bound on rows; d_n (nullable) =
+// device-resident actual row count (<= n_max) produced by a previous pass.
+int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
+                       int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                       cudaStream_t s);
+
+// Fused or unfused chain (validated arguments); used by the C-ABI and fission.
+int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,
+                      int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                      size_t ws_bytes, cudaStream_t s);
+
+// --------------------------------------------------------------- Q1
+int launch_q1(const ra_lineitem& cols, int64_t n, int32_t cutoff, ra_q1_partial* d_partial,
+              void* d_ws, size_t ws_bytes, cudaStream_t s);
+size_t q1_ws_bytes();
+
+}  // namespace ra
+
+// ------------------------------------------------------ device helpers
+namespace ra {
+namespace dev {
+
+__device__ __forceinline__ int4 ld_stream_v4(const int4* p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void st_relaxed_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void st_relaxed_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ int64_t ld_relaxed_s64(const int64_t* p) {
+  int64_t v;
+  asm volatile("ld.relaxed.gpu.global.s64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// acq_rel fetch-add: orders this CTA's earlier header reads before the ticket.
+__device__ __forceinline__ uint32_t atom_add_acq_rel_u32(uint32_t* p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+
+__device__ __forceinline__ int64_t warp_sum_s64(int64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+}  // namespace dev
+}  // namespace ra

@@ -1,0 +1,585 @@
+// select_fused.cu — single-pass fused SELECT (chain) for sm_100a.
+//
+// The paper's SELECT has four stages — partition, filter, buffer, gather —
+// in two CUDA kernels separated by a global synchronisation so that each CTA
+// can find "the correct position in the final array" of its matches
+// (Fig 3).  Fusing a chain inserts further filter
+// stages after the first and keeps one partition/buffer/gather
+// (Fig 6; L784-785, L812-814).
+//
+// Here the whole chain is ONE persistent, warp-specialised kernel: two CTAs per
+// SM, each with 8 compute warps and one look-back warp.
+//
+//   partition  4096-row tiles dealt round-robin (tile i of CTA b is b + i*G,
+//              G = grid); the grid is launched cooperatively, so every CTA is
+//              co-resident (a CTA may wait on any lower tile).
+//   load       each tile arrives by one 1-D bulk async copy (cp.async.bulk, TMA
+//              engine) into a 3-slot shared-memory ring completed on mbarriers;
+//              the copies of the next two tiles are always in flight.
+//   filter     each compute warp owns 512 contiguous rows of the tile, read as
+//              four conflict-free 128-bit shared loads per lane; the folded
+//              predicate (lo <= x <= hi, x != ne[]) is evaluated in registers.
+//   buffer     a packed 5-step warp scan and a warp-count reduction order the
+//              matches; they are compacted into a 52 KB shared-memory ring of
+//              selected rows (variable size per tile) and the tile aggregate is
+//              published at once.
+//   gather     once the look-back warp has placed a tile (its global offset),
+//              the compute warps copy its run from the ring to the output with
+//              coalesced stores.
+//
+// Look-back, B200 style.  An L2 round trip under full HBM load (~1.4 us) is
+// about two tiles' time budget, so nothing on the compute path waits for one:
+//   * exclusive(t) = inclusive(t - G) + the G-1 aggregates in between.  The
+//     CTA owns t - G and keeps its inclusive prefix, so only aggregates are
+//     read, each published in its owner's count phase — never the result of
+//     another CTA's look-back: there is no chain of dependent look-backs.
+//   * the look-back warp bulk-copies tile k's window of G-1 aggregates into
+//     shared memory when this CTA counts tile k+2 (lower CTAs have published
+//     round k by then) and resolves it at tile k+4; a word still unpublished
+//     (a lagging CTA) is re-polled individually.
+//   * compute warps write tile k at tile k+5, or earlier when the ring of
+//     selected rows runs short (high selectivity).  The ring holds only
+//     selected rows, so at 25% selectivity it is ~13 tiles deep.
+//
+// Status words carry a 28-bit launch epoch (header word bumped by the last
+// tile), so stale words of earlier launches read as "not ready": no per-call
+// memset and no second kernel.  A workspace must be re-zeroed once per 2^28
+// launches (ra_workspace_init).
+
+#include <stdio.h>
+
+#include "ra_internal.cuh"
+
+namespace ra {
+
+#ifdef RA_SEL_PROFILE  // counters for scripts/micro/sel_prof.cu; never in the product build
+__device__ unsigned long long g_sel_prof[8];
+#define PROF_ADD(k, v) atomicAdd(&g_sel_prof[k], (unsigned long long)(v))
+#else
+#define PROF_ADD(k, v)
+#endif
+
+namespace {
+
+// status word: [63:62] flag | [61:34] epoch tag | [33:0] aggregate
+constexpr uint64_t FLAG_A = 1ull << 62;  // tile aggregate published
+constexpr int TAG_SHIFT = 34;
+constexpr uint64_t TAG_MASK = (1ull << 28) - 1;
+
+constexpr int H_EPOCH = 0;  // header word (uint32)
+
+constexpr int NW = SEL_THREADS / 32;     // compute warps
+constexpr int WROWS = SEL_TILE / NW;     // contiguous rows owned by a compute warp (512)
+constexpr int BLOCK = SEL_THREADS + 32;  // + the look-back warp
+constexpr int K = SEL_LAG + 2;           // metadata slots: tiles counted but not yet written
+constexpr int D1 = 2;                    // window of tile k copied when tile k+D1 is counted
+constexpr int D2 = 4;                    // ... and resolved when tile k+D2 is counted
+constexpr int Q = D2 - D1 + 1;           // window slots
+constexpr int LBW = 10;                  // window words per lane: 320 >= G-1
+constexpr int WIN_WORDS = 32 * LBW;      // window slot capacity (words)
+constexpr int MAX_GRID = WIN_WORDS - 2;  // window of G-1 words + alignment slack
+static_assert(SEL_VEC == 4, "rows per lane are packed as 4 x 8-bit counts");
+static_assert(NW <= 32, "one warp reduces the per-warp counts");
+static_assert(SEL_LAG >= D2 + 1, "a tile is placed before it is due");
+static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");
+
+struct SelParams {
+  const int32_t* abase;  // 16-B aligned base, = d_in - mis
+  int64_t n;             // host bound on rows
+  const int64_t* d_n;    // optional device row count (unfused passes)
+  int32_t* out;
+  int64_t out_cap;
+  int64_t* d_count;
+  uint32_t* hdr;
+  uint64_t* status;  // status[tile]
+  int32_t mis;       // rows of d_in's 16-B chunk before d_in (0..3)
+  int32_t lo, hi;
+  int32_t n_ne;
+  int32_t ne[RA_MAX_PREDS];
+};
+
+struct __align__(128) SelSmem {
+  int4 in[SEL_INSLOTS][SEL_TILE / 4];  // input tiles (bulk-copy destination)
+  int32_t ring[SEL_OUTRING];           // selected rows of counted, not yet written tiles
+  uint64_t win[Q][WIN_WORDS];          // look-back windows (bulk-copied status words)
+  uint64_t full[SEL_INSLOTS];          // TMA -> compute: tile landed
+  uint64_t winfull[Q];                 // TMA -> look-back: window landed
+  uint64_t counted[K];                 // compute -> look-back: aggregate in cnt[]
+  uint64_t placed[K];                  // look-back -> compute: offset in goff[]
+  uint32_t wtot[2][NW];                // per-warp selected counts (double-buffered by tile)
+  int32_t cnt[K];                      // tile aggregates
+  int32_t start[K];                    // tile run start in the ring (mod SEL_OUTRING)
+  int64_t goff[K];                     // tile output offsets
+  int64_t n;
+  uint32_t epoch;
+  int32_t demand;  // oldest tile the compute warps are waiting to write (-1: none yet)
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// Compute warps synchronise among themselves only (named barrier 1).
+__device__ __forceinline__ void compute_bar() { asm volatile("bar.sync 1, %0;" ::"n"(SEL_THREADS) : "memory"); }
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <bool HAS_NE>
+__device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
+  bool k = (x >= P.lo) & (x <= P.hi);
+  if (HAS_NE) {
+#pragma unroll
+    for (int j = 0; j < RA_MAX_PREDS; ++j)
+      if (j < P.n_ne) k &= (x != P.ne[j]);
+  }
+  return k;
+}
+
+__device__ __forceinline__ int32_t comp(const int4& v, int c) {
+  return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+
+// Issue the bulk copy of tile t into input slot s (one thread).
+__device__ __forceinline__ void issue_tile(SelSmem& S, const SelParams& P, int64_t nv, int64_t t, int s) {
+  const int64_t v0 = t * SEL_TILE;
+  int64_t rows = nv - v0;
+  if (rows > SEL_TILE) rows = SEL_TILE;
+  const uint32_t bytes = (uint32_t)((rows * 4 + 15) & ~15ll);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // the slot was last read by generic loads
+  mbar_arrive_expect_tx(&S.full[s], bytes);
+  bulk_g2s(&S.in[s][0], P.abase + v0, bytes, &S.full[s]);
+}
+
+// Look-back warp: bulk-copy the window of tile tp — status[tp-G+1 .. tp-1] —
+// into window slot q (16-B aligned start: one extra word may precede it).
+__device__ __forceinline__ void issue_window(SelSmem& S, const SelParams& P, int64_t tp, int64_t G, int q) {
+  int64_t s0 = tp - G + 1;
+  if (s0 < 0) s0 = 0;
+  s0 &= ~1ll;
+  const uint32_t bytes = (uint32_t)(((tp - s0) * 8 + 15) & ~15ll);
+  if (bytes == 0) {  // tile 0: nothing to read
+    mbar_arrive(&S.winfull[q]);
+    return;
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  mbar_arrive_expect_tx(&S.winfull[q], bytes);
+  bulk_g2s(&S.win[q][0], P.status + s0, bytes, &S.winfull[q]);
+}
+
+// Sum of the aggregates in tile tp's window (one warp).  An aggregate is
+// <= SEL_TILE < 2^32, so a word published by this launch has its high half
+// exactly `want` = (FLAG_A | tag) >> 32: readiness is one compare and the sum
+// fits 32 bits (one REDUX).  Words still unpublished in the copy are re-polled.
+__device__ __forceinline__ uint32_t window_sum(const SelSmem& S, const SelParams& P, int64_t tp, int64_t G, int q,
+                                               int lane, uint32_t want) {
+  int64_t lo = tp - G + 1;
+  if (lo < 0) lo = 0;
+  const int64_t s0 = lo & ~1ll;
+  uint64_t w[LBW];
+#pragma unroll
+  for (int c = 0; c < LBW; ++c) {
+    const int64_t idx = lo + LBW * lane + c;  // tile whose aggregate this word is
+    w[c] = idx < tp ? S.win[q][idx - s0] : ((uint64_t)want << 32);
+  }
+  for (int spins = 0;; ++spins) {
+    bool missing = false;
+#pragma unroll
+    for (int c = 0; c < LBW; ++c) missing |= (uint32_t)(w[c] >> 32) != want;
+    if (!__any_sync(0xffffffffu, missing)) break;
+    if (lane == 0) PROF_ADD(0, 1);
+    if (spins > 1) __nanosleep(64);
+#pragma unroll
+    for (int c = 0; c < LBW; ++c)
+      if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + lo + LBW * lane + c);
+  }
+  uint32_t v = 0;
+#pragma unroll
+  for (int c = 0; c < LBW; ++c) v += (uint32_t)w[c];
+  return __reduce_add_sync(0xffffffffu, v);
+}
+
+// Compute warps: copy tile k's run of selected rows from the ring to its place.
+__device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k, int tid) {
+  if (tid == 0) *(volatile int*)&S.demand = k;  // tell the look-back warp not to wait for later counts
+  mbar_wait(&S.placed[k % K], (uint32_t)((k / K) & 1));
+  const int64_t g = S.goff[k % K];
+  const int32_t c = S.cnt[k % K];
+  const int32_t* run = S.ring + S.start[k % K];  // contiguous, never wraps
+  int64_t lim = P.out_cap - g;
+  lim = lim < 0 ? 0 : (lim > c ? c : lim);
+  int32_t* __restrict__ out = P.out + g;
+  for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = run[e];
+}
+
+template <bool HAS_NE>
+__global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams P) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  SelSmem& S = *reinterpret_cast<SelSmem*>(smem_raw);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+
+  if (tid == 0) {
+    int64_t n = P.n;
+    if (P.d_n) {
+      const int64_t dn = dev::ld_relaxed_s64(P.d_n);
+      n = dn < n ? (dn < 0 ? 0 : dn) : n;
+    }
+    S.n = n;
+    S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);
+    S.demand = -1;
+    for (int s = 0; s < SEL_INSLOTS; ++s) mbar_init(&S.full[s], 1);
+    for (int s = 0; s < Q; ++s) mbar_init(&S.winfull[s], 1);
+    for (int s = 0; s < K; ++s) {
+      mbar_init(&S.counted[s], 1);
+      mbar_init(&S.placed[s], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const int64_t n = S.n;
+  const int64_t nv = n + P.mis;  // virtual rows, counted from the aligned base
+  const int64_t ntiles = n > 0 ? (nv + SEL_TILE - 1) / SEL_TILE : 0;
+  const uint64_t tag = S.epoch & TAG_MASK;
+  const int64_t G = gridDim.x;
+  const int64_t b = blockIdx.x;
+  const int m = ntiles > b ? (int)((ntiles - b + G - 1) / G) : 0;  // tiles of this CTA
+  if (ntiles == 0) {
+    if (b == 0 && tid == 0) *P.d_count = 0;
+    return;
+  }
+
+  if (warp == NW) {
+    // ======================= look-back warp: tile offsets =======================
+    const uint32_t want = (uint32_t)((FLAG_A | (tag << TAG_SHIFT)) >> 32);
+    int64_t my_prefix = 0;  // inclusive prefix of this CTA's last placed tile
+    // Tile k's window is copied once tile k+D1 is counted and resolved once
+    // tile k+D2 is counted — or at once when the compute warps already wait
+    // for tile k (`demand`, ring of selected rows full at high selectivity).
+    auto due = [&](int k, int d) {
+      const int x = k + d;
+      if (x >= m) return true;
+      if (*(volatile int*)&S.demand >= k) return true;
+      return mbar_test(&S.counted[x % K], (uint32_t)((x / K) & 1));
+    };
+    int c_next = 0;  // next window to copy
+    for (int k = 0; k < m; ++k) {
+      for (int spins = 0;; ++spins) {
+        if (c_next < m && c_next < k + Q && due(c_next, D1)) {
+          if (lane == 0) issue_window(S, P, b + (int64_t)c_next * G, G, c_next % Q);
+          ++c_next;
+          continue;
+        }
+        if (c_next > k && due(k, D2)) break;
+        if (spins > 2) __nanosleep(128);
+      }
+      {  // resolve tile k
+        const int64_t tp = b + (int64_t)k * G;
+        mbar_wait(&S.counted[k % K], (uint32_t)((k / K) & 1));  // own aggregate in cnt[]
+        mbar_wait(&S.winfull[k % Q], (uint32_t)((k / Q) & 1));
+        const uint32_t sum = window_sum(S, P, tp, G, k % Q, lane, want);
+        const int64_t g = my_prefix + (int64_t)sum;
+        my_prefix = g + S.cnt[k % K];
+        if (lane == 0) {
+          S.goff[k % K] = g;
+          if (tp == ntiles - 1) {  // every tile has published (read the epoch): advance it
+            *P.d_count = my_prefix;
+            st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
+          }
+          mbar_arrive(&S.placed[k % K]);
+        }
+        __syncwarp();
+      }
+    }
+    return;
+  }
+
+  // ======================= compute warps ======================================
+  if (tid == 0)
+    for (int s = 0; s < SEL_AHEAD && s < m; ++s) issue_tile(S, P, nv, b + (int64_t)s * G, s);
+
+  int32_t wp = 0;  // end of the newest run in the ring
+  int head = 0;    // oldest tile not yet written
+  for (int i = 0; i < m; ++i) {
+    // ---- filter tile i
+    const int slot = i % SEL_INSLOTS;
+#ifdef RA_SEL_PROFILE
+    const long long c0 = clock64();
+#endif
+    mbar_wait(&S.full[slot], (uint32_t)((i / SEL_INSLOTS) & 1));
+#ifdef RA_SEL_PROFILE
+    if (tid == 0) PROF_ADD(2, clock64() - c0);
+#endif
+    const int64_t t = b + (int64_t)i * G;
+    int4 v[SEL_VEC];
+    {
+      const int4* base = &S.in[slot][warp * (WROWS / 4)];
+#pragma unroll
+      for (int j = 0; j < SEL_VEC; ++j) v[j] = base[32 * j + lane];
+    }
+    const int64_t v0 = t * SEL_TILE + warp * WROWS;
+    uint32_t fl = 0;  // bit 4j+c: row warp*512 + 4*(32j + lane) + c selected
+    if (v0 >= P.mis && v0 + WROWS <= nv) {
+#pragma unroll
+      for (int j = 0; j < SEL_VEC; ++j)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) fl |= (uint32_t)keep<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
+    } else {
+#pragma unroll
+      for (int j = 0; j < SEL_VEC; ++j) {
+        const int64_t e0 = v0 + 4 * (32 * j + lane);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          const bool k = keep<HAS_NE>(comp(v[j], c), P) & (e0 + c >= P.mis) & (e0 + c < nv);
+          fl |= (uint32_t)k << (4 * j + c);
+        }
+      }
+    }
+    // ---- buffer: order (warp, j, lane, c); packed per-row counts, warp scan
+    uint32_t packed = 0;
+#pragma unroll
+    for (int j = 0; j < SEL_VEC; ++j) packed |= (uint32_t)__popc((fl >> (4 * j)) & 0xFu) << (8 * j);
+    uint32_t inc = packed;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, d);
+      if (lane >= d) inc += y;
+    }
+    const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);  // per-row warp totals (<= 128 each)
+    const uint32_t wtotal = (tot & 0xFF) + ((tot >> 8) & 0xFF) + ((tot >> 16) & 0xFF) + (tot >> 24);
+    if (lane == 0) S.wtot[i & 1][warp] = wtotal;
+    compute_bar();  // B1: wtot visible; tile i-1's input slot is free
+    if (tid == 0 && i + SEL_AHEAD < m)
+      issue_tile(S, P, nv, b + (int64_t)(i + SEL_AHEAD) * G, (i + SEL_AHEAD) % SEL_INSLOTS);
+    const uint32_t wt = lane < NW ? S.wtot[i & 1][lane] : 0u;
+    const int32_t agg = (int32_t)__reduce_add_sync(0xffffffffu, wt);
+    const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
+    if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
+      dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
+      S.cnt[i % K] = agg;
+      mbar_arrive(&S.counted[i % K]);
+    }
+    // ---- allocate the tile's run: contiguous in the ring (a run that does not
+    // fit before the end starts again at 0); write the oldest tiles early if
+    // the ring is short.  Every thread takes the same decisions.
+    int32_t start;
+    bool forced = false;
+    while (true) {
+      if (head == i) {  // nothing pending
+        start = 0;
+        break;
+      }
+      const int32_t rp = S.start[head % K];  // pending rows occupy [rp, wp) circularly
+      if (rp <= wp) {
+        if (wp + agg <= SEL_OUTRING) { start = wp; break; }
+        if (agg <= rp) { start = 0; break; }
+      } else if (wp + agg <= rp) {
+        start = wp;
+        break;
+      }
+      write_tile(S, P, head, tid);
+      ++head;
+      forced = true;
+    }
+    if (forced) compute_bar();  // rows written out are read before they are overwritten
+    if (tid == 0) S.start[i % K] = start;
+    // ---- scatter tile i into the ring
+    {
+      const uint32_t ex = inc - packed;
+      int32_t rb = start + wbase;
+#pragma unroll
+      for (int j = 0; j < SEL_VEC; ++j) {
+        int32_t p = rb + (int32_t)((ex >> (8 * j)) & 0xFFu);
+        const uint32_t bits = (fl >> (4 * j)) & 0xFu;
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+          if (bits & (1u << c)) S.ring[p++] = comp(v[j], c);
+        rb += (int32_t)((tot >> (8 * j)) & 0xFFu);
+      }
+    }
+    wp = start + agg;
+    // ---- gather: tile i - SEL_LAG is due
+    if (i - SEL_LAG >= head) {
+#ifdef RA_SEL_PROFILE
+      const long long c1 = clock64();
+#endif
+      write_tile(S, P, head, tid);
+#ifdef RA_SEL_PROFILE
+      if (tid == 0) { PROF_ADD(1, clock64() - c1); PROF_ADD(3, 1); }
+#endif
+      ++head;
+    }
+  }
+  compute_bar();  // scatters of the last tiles are visible
+  for (; head < m; ++head) write_tile(S, P, head, tid);
+}
+
+struct KernelCfg {
+  int grid_per_sm[64][2];
+};
+KernelCfg g_cfg;
+
+template <bool HAS_NE>
+int ensure_config(int dev, int& per_sm) {
+  int& c = g_cfg.grid_per_sm[dev][HAS_NE ? 1 : 0];
+  if (!c) {
+    const int smem = (int)sizeof(SelSmem);
+    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(select smem)");
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE>, BLOCK, smem);
+    if (e != cudaSuccess) return cuda_fail(e, "occupancy(select)");
+    if (occ < 1) return fail(RA_E_CUDA, "select kernel does not fit on an SM");
+    c = occ;
+  }
+  per_sm = c;
+  return RA_OK;
+}
+
+}  // namespace
+
+int64_t sel_max_tiles(int64_t n) { return (n + 3 + SEL_TILE - 1) / SEL_TILE + 1; }
+
+size_t sel_status_bytes(int64_t n) { return SEL_HDR_BYTES + 8 * (size_t)sel_max_tiles(n) + 16; }
+
+size_t sel_inter_bytes(int64_t n) {
+  // two int32[n] relations + two int64 counts, 256-B granules
+  const size_t rel = (((size_t)(n > 0 ? n : 1) * 4 + 255) / 256) * 256;
+  return 2 * rel + 256;
+}
+
+int sel_ctas_per_sm() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  int per_sm = 0;
+  if (ensure_config<false>(dev, per_sm)) return -1;
+  return per_sm;
+}
+
+int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
+                       int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                       cudaStream_t s) {
+  SelParams P;
+  const uintptr_t a = (uintptr_t)d_in;
+  P.mis = (int32_t)((a & 15u) >> 2);
+  P.abase = (const int32_t*)(a - (a & 15u));
+  P.n = n_max;
+  P.d_n = d_n;
+  P.out = d_out;
+  P.out_cap = out_cap;
+  P.d_count = d_count;
+  P.hdr = (uint32_t*)d_ws;
+  P.status = (uint64_t*)((char*)d_ws + SEL_HDR_BYTES);
+  P.lo = cp.lo;
+  P.hi = cp.hi;
+  P.n_ne = cp.n_ne;
+  for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne[j] = j < cp.n_ne ? cp.ne[j] : 0;
+  if (n_max >= ((int64_t)1 << 34)) return fail(RA_E_INVAL, "n=%lld >= 2^34", (long long)n_max);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  const bool ne = cp.n_ne > 0;
+  int per_sm = 1;
+  int rc = ne ? ensure_config<true>(dev, per_sm) : ensure_config<false>(dev, per_sm);
+  if (rc) return rc;
+  const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
+  int64_t grid = (int64_t)num_sms() * per_sm;
+  if (grid > ntiles_max) grid = ntiles_max;
+  if (grid > MAX_GRID) grid = MAX_GRID;
+  if (grid < 1) grid = 1;
+  // Cooperative launch: the driver guarantees all CTAs are co-resident, which
+  // the static tile assignment needs (a CTA may wait on any lower tile).
+  const size_t smem = sizeof(SelSmem);
+  void* args[] = {(void*)&P};
+  cudaError_t le = cudaLaunchCooperativeKernel(
+      ne ? (const void*)select_fused_kernel<true> : (const void*)select_fused_kernel<false>,
+      dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
+  if (le != cudaSuccess) return cuda_fail(le, "select_fused_kernel cooperative launch");
+  count_launch();
+  return RA_OK;
+}
+
+int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,
+                      int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                      size_t ws_bytes, cudaStream_t s) {
+  if (fused || k <= 1) {
+    CanonPred cp;
+    int rc = canonicalize(h_preds, k, &cp);
+    if (rc) return rc;
+    return launch_select_pass(d_in, n, nullptr, cp, d_out, out_cap, d_count, d_ws, s);
+  }
+  // Unfused composition: one pass per predicate, intermediates at the end of
+  // the workspace (disjoint from any status words this workspace can hold).
+  const size_t rel = (((size_t)(n > 0 ? n : 1) * 4 + 255) / 256) * 256;
+  char* inter = (char*)d_ws + ws_bytes - sel_inter_bytes(n);
+  int32_t* buf[2] = {(int32_t*)inter, (int32_t*)(inter + rel)};
+  int64_t* cnt = (int64_t*)(inter + 2 * rel);
+  const int32_t* src = d_in;
+  const int64_t* src_n = nullptr;
+  for (int j = 0; j < k; ++j) {
+    CanonPred cp;
+    int rc = canonicalize(&h_preds[j], 1, &cp);
+    if (rc) return rc;
+    const bool last = (j == k - 1);
+    int32_t* dst = last ? d_out : buf[j & 1];
+    int64_t* dcnt = last ? d_count : &cnt[j & 1];
+    rc = launch_select_pass(src, n, src_n, cp, dst, last ? out_cap : n, dcnt, d_ws, s);
+    if (rc) return rc;
+    src = dst;
+    src_n = dcnt;
+  }
+  return RA_OK;
+}
+
+}  // namespace ra

@@ -1,0 +1,45 @@
+"""Small driver for ncu: runs the hot-path kernels a few times at bench sizes.
+
+usage: python scripts/prof_driver.py {select|unfused|q1|select1m} [reps] [log2n] [k] [sel]
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_ipps_wudwcyc12_b200 as R  # noqa: E402
+import ragen  # noqa: E402
+
+
+def main():
+    what = sys.argv[1]
+    reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
+    log2n = int(sys.argv[3]) if len(sys.argv) > 3 else 28
+    k = int(sys.argv[4]) if len(sys.argv) > 4 else 2
+    sel = float(sys.argv[5]) if len(sys.argv) > 5 else 0.5
+    torch.cuda.set_device(0)
+    if what in ("select", "unfused", "select1m"):
+        n = 1 << (20 if what == "select1m" else log2n)
+        x = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(2, x)
+        preds = [("lt", t) for t in ragen.nested_thresholds(sel, k)] if what != "select1m" else [("lt", 0)]
+        out = torch.empty(n, dtype=torch.int32, device="cuda")
+        for _ in range(reps):
+            R.select_chain(x, preds, fused=(what != "unfused"), out=out)
+    elif what == "q1":
+        n = ragen.rows_for_sf(10)
+        cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+                for name, dt in ragen.LINEITEM_COLUMNS}
+        ragen.lineitem_dev(5, ragen.parts_for_sf(10), cols)
+        for _ in range(reps):
+            R.q1(cols)
+    torch.cuda.synchronize()
+    print("done", what)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,115 @@
+"""C-ABI checks that need no GPU: libra.so loads, exports every entry point
+include/ra.h declares, sizes workspaces, rejects bad arguments before touching
+CUDA, and its host-side Q1 finalize merges partials exactly (fed with partials
+assembled from the oracle's exact group sums)."""
+import ctypes
+import subprocess
+
+import numpy as np
+import pytest
+
+import oracle
+import ragen
+
+R = pytest.importorskip("paper_conf_ipps_wudwcyc12_b200")
+
+
+def test_exports_every_header_symbol():
+    declared = R.exported_symbols_from_header()
+    assert len(declared) >= 12
+    nm = subprocess.run(["nm", "-D", "--defined-only", R.LIB_PATH], capture_output=True, text=True).stdout
+    exported = {line.split()[-1] for line in nm.splitlines() if " T " in line}
+    assert set(declared) <= exported, set(declared) - exported
+    assert {s for s in exported if s.startswith("ra_")} == set(declared)
+
+
+def test_struct_sizes_match_header_layout():
+    assert ctypes.sizeof(R.ra_pred) == 8
+    assert ctypes.sizeof(R.ra_q1_group) == 64
+    assert ctypes.sizeof(R.ra_q1_partial) == 16 + 6 * 64
+    assert ctypes.sizeof(R.ra_q1_row) == 8 + 8 * 8 + 3 * 8
+    assert R.ra_version() == 1
+
+
+def test_workspace_sizes():
+    assert R.ra_select_workspace_bytes(0, 1, 1) >= 256
+    f = R.ra_select_workspace_bytes(1 << 28, 2, 1)
+    u = R.ra_select_workspace_bytes(1 << 28, 2, 0)
+    assert f < 2 << 20  # status words only: ~16 B per 4096-row tile
+    assert u >= f + 2 * 4 * (1 << 28)  # two device-resident intermediates
+    assert R.ra_select_workspace_bytes(1 << 28, 1, 0) == f  # k=1 never materialises
+    assert R.ra_fission_workspace_bytes(1 << 20, 3, 2, 1) >= 3 * 2 * 4 * (1 << 20)
+    assert R.ra_fission_workspace_bytes(0, 3, 2, 1) == 0
+
+
+def test_argument_errors_without_gpu():
+    P = R.make_preds([("lt", 0)])
+    with pytest.raises(R.RAError) as e:  # null count
+        R.ra_select_chain(0, 10, P, 1, 1, 0, 10, 0, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:  # k > 8
+        R.ra_select_chain(0, 0, R.make_preds([("lt", 0)] * 9), 9, 1, 0, 0, 8, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:  # workspace too small
+        R.ra_select_chain(4096, 1 << 20, P, 1, 1, 4096, 1 << 20, 8, 256, 16, 0)
+    assert e.value.code == R.RA_E_WORKSPACE
+    with pytest.raises(R.RAError) as e:  # misaligned
+        R.ra_select_chain(4098, 10, P, 1, 1, 4096, 10, 8, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:  # bad op
+        R.ra_select_chain(4096, 10, R.make_preds([(17, 0)]), 1, 1, 4096, 10, 8, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    li = R.ra_lineitem()
+    with pytest.raises(R.RAError) as e:  # null columns
+        R.ra_q1(li, 5, 10471, 4096, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:  # n >= 2^32
+        R.ra_q1(li, 1 << 32, 10471, 4096, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    assert "n=" in R.ra_last_error()
+
+
+SLOT = {(ord(rf), ord(ls)): 2 * i + j for i, rf in enumerate("ANR") for j, ls in enumerate("FO")}
+
+
+def partial_from_oracle_rows(rows, status=0, nrows=0):
+    p = R.ra_q1_partial()
+    p.status, p.n_groups, p.rows = status, 6, nrows
+    for r in rows:
+        g = p.group[SLOT[(r["rf_byte"], r["ls_byte"])]]
+        g.count, g.sum_qty, g.sum_base_price, g.sum_disc = (
+            r["count_order"], r["sum_qty"], r["sum_base_price"], r["sum_disc"])
+        g.sum_disc_price_lo, g.sum_disc_price_hi = r["sum_disc_price"] & (2**64 - 1), r["sum_disc_price"] >> 64
+        g.sum_charge_lo, g.sum_charge_hi = r["sum_charge"] & (2**64 - 1), r["sum_charge"] >> 64
+    return p
+
+
+def test_finalize_merges_shards_exactly():
+    cols = ragen.lineitem(12, 400000, 200000)
+    whole, _ = oracle.q1(cols, 10471)
+    cuts = [0, 100, 150000, 400000]
+    parts = (R.ra_q1_partial * 3)()
+    for i, (a, b) in enumerate(zip(cuts[:-1], cuts[1:])):
+        rows, _ = oracle.q1({k: v[a:b] for k, v in cols.items()}, 10471)
+        parts[i] = partial_from_oracle_rows(rows)
+    got, rc = R.q1_finalize(parts)
+    assert rc == R.RA_OK
+    assert len(got) == len(whole) == 4
+    for g, w in zip(got, whole):
+        for k in ("count_order", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "sum_disc",
+                  "avg_qty", "avg_price", "avg_disc"):
+            assert g[k] == w[k], k
+
+
+def test_finalize_128bit_charge_and_domain():
+    p = R.ra_q1_partial()
+    p.group[3].count = 5
+    p.group[3].sum_charge_lo, p.group[3].sum_charge_hi = 2**64 - 1, 0
+    q = R.ra_q1_partial()
+    q.group[3].count = 1
+    q.group[3].sum_charge_lo = 1
+    q.status = 2
+    got, rc = R.q1_finalize((R.ra_q1_partial * 2)(p, q))
+    assert rc == R.RA_E_DOMAIN
+    assert got[0]["sum_charge"] == 2**64 and got[0]["count_order"] == 6
+    assert (got[0]["returnflag"], got[0]["linestatus"]) == ("N", "O")

@@ -1,0 +1,144 @@
+"""GPU parity: libra.so's fused Q1 (+ host finalize) vs the CPU oracle.
+
+Bit-exact: every group's count and scaled-integer sums (128-bit disc_price and
+charge) and the AVG doubles (C12: one division of exact operands on both
+sides), plus the domain status bits.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import ragen
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+CUTOFF = 10471
+KEYS = ("count_order", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "sum_disc",
+        "avg_qty", "avg_price", "avg_disc")
+
+
+@pytest.fixture(scope="module")
+def R():
+    import paper_conf_ipps_wudwcyc12_b200 as R
+    return R
+
+
+def to_dev(cols, offset=0):
+    out = {}
+    for k, v in cols.items():
+        pad = np.zeros(offset, dtype=v.dtype)
+        out[k] = torch.from_numpy(np.concatenate([pad, v])).cuda()[offset:]
+    return out
+
+
+def gpu_q1(R, dcols, cutoff=CUTOFF):
+    part = R.q1(dcols, cutoff)
+    torch.cuda.synchronize()
+    raw = bytes(part.cpu().numpy().tobytes())
+    rows, rc = R.q1_finalize(raw)
+    return rows, rc, R.partials_from_bytes(raw)[0]
+
+
+def assert_same(rows, exp):
+    assert [(r["returnflag"], r["linestatus"]) for r in rows] == [(e["returnflag"], e["linestatus"]) for e in exp]
+    for r, e in zip(rows, exp):
+        for k in KEYS:
+            assert r[k] == e[k], (r["returnflag"], r["linestatus"], k, r[k], e[k])
+
+
+@pytest.mark.parametrize("n", [0, 1, 3, 4, 5, 255, 256, 1023, 4097, 100003])
+@pytest.mark.parametrize("offset", [0, 1, 2, 3])
+def test_small_sizes_and_alignment(R, n, offset):
+    cols = ragen.lineitem(31 + n, n, 2000)
+    exp, st = oracle.q1(cols, CUTOFF)
+    rows, rc, part = gpu_q1(R, to_dev(cols, offset))
+    assert rc == R.RA_OK and part.status == st == 0 and part.rows == n
+    assert_same(rows, exp)
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0, 10.0])
+def test_scale_factors(R, sf):
+    n = ragen.rows_for_sf(sf)
+    cols = ragen.lineitem(3, n, ragen.parts_for_sf(sf))
+    exp, st = oracle.q1(cols, CUTOFF)
+    rows, rc, _ = gpu_q1(R, to_dev(cols))
+    assert rc == R.RA_OK and st == 0
+    assert_same(rows, exp)
+
+
+@pytest.mark.parametrize("cutoff", [8035, 8036, 9298, 10000, 10471, 10561, 2**31 - 1, -(2**31)])
+def test_cutoffs(R, cutoff):
+    cols = ragen.lineitem(4, 200001, 20000)
+    exp, _ = oracle.q1(cols, cutoff)
+    rows, rc, _ = gpu_q1(R, to_dev(cols), cutoff)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)
+
+
+def test_device_generated_sf10_launch_config(R):
+    """BASELINE configs[2] (SF10, 60 M rows) generated on the device exactly as
+    bench.py does; oracle over the same rows regenerated on the host."""
+    n = ragen.rows_for_sf(10)
+    dcols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+             for name, dt in ragen.LINEITEM_COLUMNS}
+    ragen.lineitem_dev(3, ragen.parts_for_sf(10), dcols)
+    rows, rc, _ = gpu_q1(R, dcols)
+    cols = ragen.lineitem(3, n, ragen.parts_for_sf(10))
+    exp, _ = oracle.q1(cols, CUTOFF)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)
+
+
+def test_domain_errors_reported(R):
+    cols = ragen.lineitem(5, 50000, 2000)
+    bad = {k: v.copy() for k, v in cols.items()}
+    bad["returnflag"][100] = ord("Z")
+    bad["tax"][200] = 101
+    exp, st = oracle.q1(bad, 10561)
+    assert st == 3
+    rows, rc, part = gpu_q1(R, to_dev(bad), 10561)
+    assert rc == R.RA_E_DOMAIN and part.status == st
+    # out-of-domain rows are not accumulated: equal to the oracle without them
+    keep = np.ones(50000, bool)
+    keep[[100, 200]] = False
+    exp2, _ = oracle.q1({k: v[keep] for k, v in bad.items()}, 10561)
+    assert_same(rows, exp2)
+
+
+def test_arbitrary_bytes_random(R):
+    rng = np.random.default_rng(0)
+    cols = ragen.lineitem(6, 30000, 2000)
+    idx = rng.integers(0, 30000, 50)
+    cols["linestatus"][idx] = rng.integers(0, 256, 50).astype(np.uint8)
+    exp, st = oracle.q1(cols, 10561)
+    rows, rc, part = gpu_q1(R, to_dev(cols), 10561)
+    assert part.status == st
+    assert rc == (R.RA_E_DOMAIN if st else R.RA_OK)
+
+
+def test_shard_partials_merge_exactly(R):
+    """Row-range shards -> partials -> exact slotwise merge == oracle on the whole."""
+    n = 1_000_003
+    cols = ragen.lineitem(7, n, 200000)
+    exp, _ = oracle.q1(cols, CUTOFF)
+    cuts = [0, 1, 250001, 600000, n]
+    raws = b""
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        part = R.q1(to_dev({k: v[a:b] for k, v in cols.items()}), CUTOFF)
+        torch.cuda.synchronize()
+        raws += part.cpu().numpy().tobytes()
+    rows, rc = R.q1_finalize(raws)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)
+
+
+def test_repeated_launches_self_clean(R):
+    cols = ragen.lineitem(8, 300000, 20000)
+    exp, _ = oracle.q1(cols, CUTOFF)
+    d = to_dev(cols)
+    parts = [R.q1(d, CUTOFF) for _ in range(20)]
+    torch.cuda.synchronize()
+    for p in parts:
+        rows, rc = R.q1_finalize(bytes(p.cpu().numpy().tobytes()))
+        assert_same(rows, exp)

@@ -1,0 +1,163 @@
+"""GPU parity: libra.so's fused / unfused SELECT chain vs the CPU oracle.
+
+Bit-exact comparison of the selected values (order-preserving, unique result)
+and of the count, on seeded inputs from ragen; sizes span several 4096-row
+tiles, ragged tails, misaligned starts, and BASELINE's 2^20 / 2^28 configs.
+"""
+import numpy as np
+import pytest
+from hypothesis import given, settings, strategies as st
+
+import oracle
+import ragen
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def R():
+    import paper_conf_ipps_wudwcyc12_b200 as R
+    return R
+
+
+def run(R, x_np, preds, fused=True, offset=0, out_cap=None):
+    xt = torch.from_numpy(np.concatenate([np.zeros(offset, np.int32), x_np])).cuda()
+    x = xt[offset:]
+    out = None
+    if out_cap is not None:
+        out = torch.full((max(1, out_cap),), -7, dtype=torch.int32, device="cuda")
+    o, c = R.select_chain(x, preds, fused=fused, out=out)
+    torch.cuda.synchronize()
+    c = int(c.item())
+    return o.cpu().numpy(), c
+
+
+SIZES = [0, 1, 3, 4, 5, 4095, 4096, 4097, 8191, 12289, 100003, 1 << 20]
+
+
+@pytest.mark.parametrize("n", SIZES)
+@pytest.mark.parametrize("offset", [0, 1, 3])
+def test_single_select_sizes_and_alignment(R, n, offset):
+    x = ragen.int32_column(100 + n, n)
+    preds = [("lt", 0)]
+    exp = oracle.select(x, preds)
+    got, c = run(R, x, preds, offset=offset)
+    assert c == exp.size
+    np.testing.assert_array_equal(got[:c], exp)
+
+
+@pytest.mark.parametrize("s", [0.01, 0.1, 0.25, 0.5, 0.75, 0.9])
+@pytest.mark.parametrize("k", [1, 2, 3])
+@pytest.mark.parametrize("fused", [True, False])
+def test_nested_chain_selectivity_sweep(R, s, k, fused):
+    n = (1 << 20) + 777
+    x = ragen.int32_column(2, n)
+    preds = [("lt", t) for t in ragen.nested_thresholds(s, k)]
+    exp = oracle.select(x, preds)
+    got, c = run(R, x, preds, fused=fused)
+    assert c == exp.size
+    np.testing.assert_array_equal(got[:c], exp)
+
+
+OPS = ["lt", "le", "gt", "ge", "eq", "ne"]
+
+
+@settings(max_examples=60, deadline=None)
+@given(preds=st.lists(st.tuples(st.sampled_from(OPS), st.integers(-6, 6)), max_size=8),
+       n=st.integers(0, 20000), seed=st.integers(0, 1000), fused=st.booleans())
+def test_random_chains_small_domain(R, preds, n, seed, fused):
+    """Values in [-8, 8] so EQ/NE and range folding all matter."""
+    rng = np.random.default_rng(seed)
+    x = rng.integers(-8, 9, n).astype(np.int32)
+    exp = oracle.select(x, preds)
+    got, c = run(R, x, preds, fused=fused, offset=seed % 4)
+    assert c == exp.size
+    np.testing.assert_array_equal(got[:c], exp)
+
+
+@pytest.mark.parametrize("preds", [
+    [("lt", -(2**31))], [("gt", 2**31 - 1)], [("ge", -(2**31))], [("le", 2**31 - 1)], [],
+    [("eq", -(2**31))], [("ne", 2**31 - 1), ("ne", -(2**31))], [("gt", 5), ("lt", 5)],
+    [("ge", 0), ("le", 0), ("ne", 0)], [("gt", -(10**9)), ("lt", 10**9), ("ne", 3), ("ne", 4)],
+])
+def test_extreme_predicates(R, preds):
+    x = ragen.int32_column(9, 50000)
+    x[:6] = [-(2**31), 2**31 - 1, 0, 3, 4, 5]
+    exp = oracle.select(x, preds)
+    for fused in (True, False):
+        got, c = run(R, x, preds, fused=fused)
+        assert c == exp.size
+        np.testing.assert_array_equal(got[:c], exp)
+
+
+def test_selectivity_zero_one_identity(R):
+    x = ragen.int32_column(4, 300001)
+    got, c = run(R, x, [("lt", -(2**31))])
+    assert c == 0
+    got, c = run(R, x, [])
+    assert c == x.size
+    np.testing.assert_array_equal(got[:c], x)
+
+
+def test_out_cap_truncates_but_counts(R):
+    x = ragen.int32_column(5, 100000)
+    preds = [("lt", 0)]
+    exp = oracle.select(x, preds)
+    got, c = run(R, x, preds, out_cap=1000)
+    assert c == exp.size
+    np.testing.assert_array_equal(got[:1000], exp[:1000])
+
+
+def test_workspace_reuse_across_sizes(R):
+    """Self-cleaning status words: successive calls with varying n on one workspace."""
+    for i, n in enumerate([1 << 20, 5, 0, 70000, 1 << 18, 1, (1 << 20) + 3, 4096, 0, 123457]):
+        x = ragen.int32_column(1000 + i, n)
+        preds = [("ge", -(2**30)), ("lt", 2**29)]
+        exp = oracle.select(x, preds)
+        got, c = run(R, x, preds)
+        assert c == exp.size, (i, n)
+        np.testing.assert_array_equal(got[:c], exp)
+
+
+def test_many_back_to_back_calls_same_stream(R):
+    n = 1 << 16
+    x = torch.from_numpy(ragen.int32_column(77, n)).cuda()
+    preds = [("lt", 0)]
+    exp = oracle.select(x.cpu().numpy(), preds)
+    outs = [R.select_chain(x, preds) for _ in range(50)]
+    torch.cuda.synchronize()
+    for o, c in outs:
+        assert int(c.item()) == exp.size
+        np.testing.assert_array_equal(o[: exp.size].cpu().numpy(), exp)
+
+
+def test_full_size_config_2_pow_28(R):
+    """BASELINE configs[1] at its full size, in the launch configuration bench.py
+    times (device-generated column, k=2, s=0.5): full comparison vs the oracle."""
+    n = 1 << 28
+    x = torch.empty(n, dtype=torch.int32, device="cuda")
+    ragen.int32_column_dev(2, x)
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 2)]
+    out, c = R.select_chain(x, preds)
+    torch.cuda.synchronize()
+    c = int(c.item())
+    xh = x.cpu().numpy()
+    np.testing.assert_array_equal(xh, ragen.int32_column(2, n))  # device gen == host gen
+    exp = oracle.select(xh, preds)
+    assert c == exp.size
+    np.testing.assert_array_equal(out[:c].cpu().numpy(), exp)
+    out2, c2 = R.select_chain(x, preds, fused=False)
+    torch.cuda.synchronize()
+    assert int(c2.item()) == c
+    assert torch.equal(out2[:c], out[:c])
+
+
+def test_bad_arguments_raise(R):
+    x = torch.zeros(10, dtype=torch.int32, device="cuda")
+    with pytest.raises(R.RAError) as e:
+        R.select_chain(x, [(9, 0)])
+    assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError):
+        R.select_chain(x, [("lt", 0)] * 9)

@@ -10,19 +10,21 @@
 // Here the whole chain is ONE persistent, warp-specialised kernel: two CTAs per
 // SM, each with 8 compute warps and one look-back warp.
 //
-//   partition  4096-row tiles dealt round-robin (tile i of CTA b is b + i*G,
+//   partition  8192-row tiles dealt round-robin (tile i of CTA b is b + i*G,
 //              G = grid); the grid is launched cooperatively, so every CTA is
 //              co-resident (a CTA may wait on any lower tile).
 //   load       each tile arrives by one 1-D bulk async copy (cp.async.bulk, TMA
-//              engine) into a 3-slot shared-memory ring completed on mbarriers;
-//              the copies of the next two tiles are always in flight.
-//   filter     each compute warp owns 512 contiguous rows of the tile, read as
-//              four conflict-free 128-bit shared loads per lane; the folded
+//              engine) into a 2-slot shared-memory ring completed on mbarriers;
+//              the next tile's copy (32 KB per CTA, 64 KB per SM) is always in
+//              flight while the current one is processed.
+//   filter     each compute warp owns 1024 contiguous rows of the tile, read as
+//              eight conflict-free 128-bit shared loads per lane; the folded
 //              predicate (lo <= x <= hi, x != ne[]) is evaluated in registers.
-//   buffer     a packed 5-step warp scan and a warp-count reduction order the
-//              matches; they are compacted into a 52 KB shared-memory ring of
-//              selected rows (variable size per tile) and the tile aggregate is
-//              published at once.
+//   buffer     packed 5-step warp scans (4 rows x 8 bits per word) and a
+//              warp-count reduction order the matches; they are compacted into a
+//              40 KB shared-memory ring of selected rows (variable size per
+//              tile, each run contiguous) and the tile aggregate is published at
+//              once.
 //   gather     once the look-back warp has placed a tile (its global offset),
 //              the compute warps copy its run from the ring to the output with
 //              coalesced stores.
@@ -38,8 +40,9 @@
 //     round k by then) and resolves it at tile k+4; a word still unpublished
 //     (a lagging CTA) is re-polled individually.
 //   * compute warps write tile k at tile k+5, or earlier when the ring of
-//     selected rows runs short (high selectivity).  The ring holds only
-//     selected rows, so at 25% selectivity it is ~13 tiles deep.
+//     selected rows runs short (high selectivity; the look-back warp then
+//     resolves on demand).  The ring holds only selected rows, so at 25%
+//     selectivity it is five tiles (~7 us) deep.
 //
 // Status words carry a 28-bit launch epoch (header word bumped by the last
 // tile), so stale words of earlier launches read as "not ready": no per-call
@@ -54,6 +57,7 @@ namespace ra {
 
 #ifdef RA_SEL_PROFILE  // counters for scripts/micro/sel_prof.cu; never in the product build
 __device__ unsigned long long g_sel_prof[8];
+__device__ unsigned long long* g_sel_trace;  // [tile] globaltimer at count
 #define PROF_ADD(k, v) atomicAdd(&g_sel_prof[k], (unsigned long long)(v))
 #else
 #define PROF_ADD(k, v)
@@ -69,7 +73,7 @@ constexpr uint64_t TAG_MASK = (1ull << 28) - 1;
 constexpr int H_EPOCH = 0;  // header word (uint32)
 
 constexpr int NW = SEL_THREADS / 32;     // compute warps
-constexpr int WROWS = SEL_TILE / NW;     // contiguous rows owned by a compute warp (512)
+constexpr int WROWS = SEL_TILE / NW;     // contiguous rows owned by a compute warp (1024)
 constexpr int BLOCK = SEL_THREADS + 32;  // + the look-back warp
 constexpr int K = SEL_LAG + 2;           // metadata slots: tiles counted but not yet written
 constexpr int D1 = 2;                    // window of tile k copied when tile k+D1 is counted
@@ -78,7 +82,8 @@ constexpr int Q = D2 - D1 + 1;           // window slots
 constexpr int LBW = 10;                  // window words per lane: 320 >= G-1
 constexpr int WIN_WORDS = 32 * LBW;      // window slot capacity (words)
 constexpr int MAX_GRID = WIN_WORDS - 2;  // window of G-1 words + alignment slack
-static_assert(SEL_VEC == 4, "rows per lane are packed as 4 x 8-bit counts");
+constexpr int NPK = SEL_VEC / 4;         // packed count words per lane (4 rows of 8 bits each)
+static_assert(SEL_VEC % 4 == 0 && SEL_VEC <= 8, "rows per lane are packed as 8-bit counts, fl has 32 bits");
 static_assert(NW <= 32, "one warp reduces the per-warp counts");
 static_assert(SEL_LAG >= D2 + 1, "a tile is placed before it is due");
 static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");
@@ -347,7 +352,8 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
   if (tid == 0)
     for (int s = 0; s < SEL_AHEAD && s < m; ++s) issue_tile(S, P, nv, b + (int64_t)s * G, s);
 
-  int32_t wp = 0;  // end of the newest run in the ring
+  int32_t wp = 0;    // end of the newest run in the ring
+  int32_t used = 0;  // selected rows of pending tiles in the ring
   int head = 0;    // oldest tile not yet written
   for (int i = 0; i < m; ++i) {
     // ---- filter tile i
@@ -385,17 +391,29 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       }
     }
     // ---- buffer: order (warp, j, lane, c); packed per-row counts, warp scan
-    uint32_t packed = 0;
+    uint32_t packed[NPK], inc[NPK], tot[NPK];  // 4 rows (j) per word, 8 bits each
 #pragma unroll
-    for (int j = 0; j < SEL_VEC; ++j) packed |= (uint32_t)__popc((fl >> (4 * j)) & 0xFu) << (8 * j);
-    uint32_t inc = packed;
+    for (int q = 0; q < NPK; ++q) {
+      packed[q] = 0;
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj)
+        packed[q] |= (uint32_t)__popc((fl >> (4 * (4 * q + jj))) & 0xFu) << (8 * jj);
+      inc[q] = packed[q];
+    }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, d);
-      if (lane >= d) inc += y;
+#pragma unroll
+      for (int q = 0; q < NPK; ++q) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc[q], d);
+        if (lane >= d) inc[q] += y;
+      }
     }
-    const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);  // per-row warp totals (<= 128 each)
-    const uint32_t wtotal = (tot & 0xFF) + ((tot >> 8) & 0xFF) + ((tot >> 16) & 0xFF) + (tot >> 24);
+    uint32_t wtotal = 0;
+#pragma unroll
+    for (int q = 0; q < NPK; ++q) {
+      tot[q] = __shfl_sync(0xffffffffu, inc[q], 31);  // per-row warp totals (<= 128 each)
+      wtotal += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
+    }
     if (lane == 0) S.wtot[i & 1][warp] = wtotal;
     compute_bar();  // B1: wtot visible; tile i-1's input slot is free
     if (tid == 0 && i + SEL_AHEAD < m)
@@ -405,6 +423,13 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
       dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
+#ifdef RA_SEL_PROFILE
+      if (g_sel_trace) {
+        unsigned long long gt;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+        g_sel_trace[t] = gt;
+      }
+#endif
       S.cnt[i % K] = agg;
       mbar_arrive(&S.counted[i % K]);
     }
@@ -414,12 +439,14 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     int32_t start;
     bool forced = false;
     while (true) {
-      if (head == i) {  // nothing pending
+      if (used == 0) {  // nothing pending (or only empty runs)
         start = 0;
         break;
       }
-      const int32_t rp = S.start[head % K];  // pending rows occupy [rp, wp) circularly
-      if (rp <= wp) {
+      // pending rows occupy [rp, wp), or [rp, end) + [0, wp) once they wrapped
+      const int32_t rp = S.start[head % K];
+      const bool wrapped = rp > wp || (rp == wp && used > 0);
+      if (!wrapped) {
         if (wp + agg <= SEL_OUTRING) { start = wp; break; }
         if (agg <= rp) { start = 0; break; }
       } else if (wp + agg <= rp) {
@@ -427,23 +454,25 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         break;
       }
       write_tile(S, P, head, tid);
+      used -= S.cnt[head % K];
       ++head;
       forced = true;
     }
     if (forced) compute_bar();  // rows written out are read before they are overwritten
     if (tid == 0) S.start[i % K] = start;
+    used += agg;
     // ---- scatter tile i into the ring
     {
-      const uint32_t ex = inc - packed;
       int32_t rb = start + wbase;
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
-        int32_t p = rb + (int32_t)((ex >> (8 * j)) & 0xFFu);
+        const uint32_t ex = inc[j >> 2] - packed[j >> 2];
+        int32_t p = rb + (int32_t)((ex >> (8 * (j & 3))) & 0xFFu);
         const uint32_t bits = (fl >> (4 * j)) & 0xFu;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
           if (bits & (1u << c)) S.ring[p++] = comp(v[j], c);
-        rb += (int32_t)((tot >> (8 * j)) & 0xFFu);
+        rb += (int32_t)((tot[j >> 2] >> (8 * (j & 3))) & 0xFFu);
       }
     }
     wp = start + agg;
@@ -456,6 +485,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
 #ifdef RA_SEL_PROFILE
       if (tid == 0) { PROF_ADD(1, clock64() - c1); PROF_ADD(3, 1); }
 #endif
+      used -= S.cnt[head % K];
       ++head;
     }
   }

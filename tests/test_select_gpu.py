@@ -92,6 +92,21 @@ def test_extreme_predicates(R, preds):
         np.testing.assert_array_equal(got[:c], exp)
 
 
+@pytest.mark.parametrize("lg", [23, 25])
+@pytest.mark.parametrize("s,k", [(0.01, 1), (0.1, 1), (0.5, 2), (0.6, 1), (0.75, 1), (0.9, 1), (1.0, 0)])
+def test_many_tiles_per_cta(R, lg, s, k):
+    """Several 8192-row tiles per CTA: exercises the ring of selected rows
+    (contiguous runs, wrap-around, early writes when it runs short) and the
+    lagged / on-demand look-back."""
+    n = (1 << lg) + 12345
+    x = ragen.int32_column(60 + lg, n)
+    preds = [("lt", t) for t in ragen.nested_thresholds(s, k)]
+    exp = oracle.select(x, preds)
+    got, c = run(R, x, preds)
+    assert c == exp.size
+    np.testing.assert_array_equal(got[:c], exp)
+
+
 def test_selectivity_zero_one_identity(R):
     x = ragen.int32_column(4, 300001)
     got, c = run(R, x, [("lt", -(2**31))])

@@ -206,8 +206,7 @@ def run_ours(args, D: Dist):
     cnt = torch.zeros(1, dtype=torch.int64, device=dev)
     ws_bytes = R.ra_select_workspace_bytes(n, k, 1)
     ws = torch.zeros(ws_bytes, dtype=torch.uint8, device=dev)
-    counts_all = torch.zeros(D.world, dtype=torch.int64, device=dev)
-    offsets = torch.zeros(D.world, dtype=torch.int64, device=dev)
+    from paper_conf_ipps_wudwcyc12_b200 import dist as rdist
     args_chain = (x.data_ptr(), n, P, k, 1, out.data_ptr(), n, cnt.data_ptr(), ws.data_ptr(), ws_bytes, sh)
 
     def chain_kernel(i):
@@ -217,8 +216,7 @@ def run_ours(args, D: Dist):
         if not kernel_done:
             chain_kernel(i)
         if D.pg:  # a9: gather per-rank counts -> exclusive scan -> global offsets
-            D.pg.all_gather_into_tensor(counts_all, cnt)
-            torch.cumsum(counts_all, 0, out=offsets)
+            rdist.exchange_counts(cnt)
 
     torch.cuda.synchronize()
     launches0 = R.ra_kernel_launches()
@@ -314,7 +312,8 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     # --- configs[2]: Q1 SF10 device-resident (N=1 only) and configs[4] SF100 sharded
     def q1_bench(sf, shard):
         N = ragen.rows_for_sf(sf)
-        lo, hi = (D.rank * N // D.world, (D.rank + 1) * N // D.world) if shard else (0, N)
+        from paper_conf_ipps_wudwcyc12_b200 import dist as rdist
+        lo, hi = rdist.shard_range(N, D.rank, D.world) if shard else (0, N)
         m = hi - lo
         cols = {name: torch.empty(m, dtype=getattr(torch, np.dtype(dt).name), device=dev)
                 for name, dt in ragen.LINEITEM_COLUMNS}
@@ -323,7 +322,7 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
         wsq_b = R.ra_q1_workspace_bytes(m)
         wsq = torch.zeros(wsq_b, dtype=torch.uint8, device=dev)
         li = R.lineitem_struct(cols)
-        parts = torch.zeros(D.world * part.numel(), dtype=torch.uint8, device=dev)
+        parts = [part]
 
         def kern(i):
             R.ra_q1(li, m, R.Q1_CUTOFF_DELTA90, part.data_ptr(), wsq.data_ptr(), wsq_b, sh)
@@ -332,10 +331,10 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
             if not kernel_done:
                 kern(i)
             if D.pg and shard:
-                D.pg.all_gather_into_tensor(parts, part)
+                parts[0] = rdist.gather_partials(part)
 
         qms, qkms = timed(torch, D, step, 50, 5, kernel_fn=kern)
-        raw = (parts if (D.pg and shard) else part).cpu().numpy().tobytes()
+        raw = parts[0].cpu().numpy().tobytes()
         rows, rc = R.q1_finalize(raw)
         ach = 38 * m / (qkms * 1e-3) / 1e9
         del cols

@@ -1,0 +1,85 @@
+"""Summarise ncu captures in gpurun_out/ into tracked profiles/ (per round).
+
+usage: python scripts/make_profiles.py ROUND
+Writes profiles/r<ROUND>_<name>.txt (key metrics, stall reasons, hottest SASS),
+profiles/r<ROUND>_launches.txt (per-kernel launch list of the bench command)
+and updates profiles/ncu_traffic.json (dram bytes per launch, read by bench.py).
+"""
+import collections
+import csv
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+RND = sys.argv[1] if len(sys.argv) > 1 else "01"
+OUT = os.path.join(ROOT, "profiles")
+os.makedirs(OUT, exist_ok=True)
+
+CAPTURES = {  # report -> (summary name, traffic key, command)
+    "prof_select": ("select_k2_s05_n28", "select_fused_k2_s0.5_n28",
+                    "python scripts/prof_driver.py select 5  (2^28 int32, k=2, s=0.5/stage)"),
+    "prof_select_s01": ("select_k1_s001_n28", "select_fused_k1_s0.01_n28",
+                        "python scripts/prof_driver.py select 5 28 1 0.01  (2^28 int32, k=1, s=0.01)"),
+    "prof_q1": ("q1_sf10", "q1_sf10", "python scripts/prof_driver.py q1 5  (SF10, 60M rows)"),
+}
+KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+        "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+        "launch__grid_size", "launch__block_size", "launch__registers_per_thread",
+        "launch__shared_mem_per_block_dynamic", "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "smsp__inst_executed.sum", "lts__t_bytes.sum"]
+
+
+def raw(rep):
+    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(out.splitlines()))
+    return dict(zip(rows[0], rows[2])), dict(zip(rows[0], rows[1]))
+
+
+def to_bytes(v, unit):
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(unit, 1)
+    return float(v.replace(",", "")) * scale
+
+
+traffic_path = os.path.join(OUT, "ncu_traffic.json")
+traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
+for rep, (name, tkey, cmd) in CAPTURES.items():
+    path = os.path.join(ROOT, "gpurun_out", rep + ".ncu-rep")
+    if not os.path.exists(path):
+        continue
+    vals, units = raw(path)
+    lines = [f"# ncu --set full --clock-control none capture, round {RND}", f"# command: {cmd}", ""]
+    for k in KEYS:
+        if k in vals:
+            lines.append(f"{k:60s} {vals[k]:>20s} {units.get(k, '')}")
+    rd = to_bytes(vals["dram__bytes_read.sum"], units["dram__bytes_read.sum"])
+    wr = to_bytes(vals["dram__bytes_write.sum"], units["dram__bytes_write.sum"])
+    traffic[tkey] = rd + wr
+    lines.append(f"{'dram bytes read+write per launch':60s} {rd + wr:20.0f} byte")
+    stalls = [(k.replace("smsp__pcsamp_warps_issue_stalled_", ""), float(v)) for k, v in vals.items()
+              if "pcsamp_warps_issue_stalled" in k and not k.endswith("not_issued")
+              and v.replace(".", "", 1).isdigit() and float(v) > 0]
+    tot = sum(s for _, s in stalls) or 1
+    lines += ["", "warp stall reasons (pc sampling):"]
+    lines += [f"  {k:28s} {s / tot * 100:5.1f}%" for k, s in sorted(stalls, key=lambda z: -z[1])[:10]]
+    open(os.path.join(OUT, f"r{RND}_{name}.txt"), "w").write("\n".join(lines) + "\n")
+    print("wrote", name)
+json.dump(traffic, open(traffic_path, "w"), indent=1, sort_keys=True)
+
+lpath = os.path.join(ROOT, "gpurun_out", "launches.csv")
+if os.path.exists(lpath):
+    rows = [r for r in csv.reader(open(lpath)) if len(r) > 5]
+    h = rows[0]
+    ki, vi = h.index("Kernel Name"), h.index("Metric Value")
+    agg = collections.OrderedDict()
+    for r in rows[1:]:
+        agg.setdefault(r[ki], []).append(float(r[vi].replace(",", "")))
+    total = sum(sum(v) for v in agg.values())
+    lines = [f"# round {RND}: ncu --metrics gpu__time_duration.sum --clock-control none -c 400",
+             "#   python bench.py --steps 20 --warmup 3 --no-extras   (cold-cache, serialised launches)",
+             "# launches  mean_ns  share_of_all  kernel"]
+    for k, v in agg.items():
+        lines.append(f"{len(v):4d}  {sum(v) / len(v):12.0f}  {sum(v) / total * 100:5.1f}%  {k[:110]}")
+    open(os.path.join(OUT, f"r{RND}_launches.txt"), "w").write("\n".join(lines) + "\n")
+    print("wrote launches")

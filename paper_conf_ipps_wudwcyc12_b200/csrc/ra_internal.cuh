@@ -38,11 +38,15 @@ int canonicalize(const ra_pred* preds, int k, CanonPred* out);
 
 // ------------------------------------------------------------ SELECT
 constexpr int SEL_THREADS = 256;  // compute threads per CTA (plus one look-back warp)
-constexpr int SEL_VEC = 8;        // int4 vectors per compute thread per tile
-constexpr int SEL_AHEAD = 1;      // tiles whose bulk copy is in flight ahead of the count
+#ifndef RA_SEL_VEC  // (overridable for scripts/micro sweeps only)
+#define RA_SEL_VEC 8
+#define RA_SEL_AHEAD 1
+#define RA_SEL_OUTRING 10240
+#endif
+constexpr int SEL_VEC = RA_SEL_VEC;      // int4 vectors per compute thread per tile
+constexpr int SEL_AHEAD = RA_SEL_AHEAD;  // tiles whose bulk copy is in flight ahead of the count
 constexpr int SEL_INSLOTS = SEL_AHEAD + 1;           // input ring slots (tiles)
-constexpr int SEL_LAG = 5;        // a tile is written SEL_LAG tiles after it is counted (or earlier)
-constexpr int SEL_OUTRING = 10240;                   // compacted-row ring (int32), 40 KB
+constexpr int SEL_OUTRING = RA_SEL_OUTRING;          // compacted-row ring (int32), 40 KB
 constexpr int SEL_TILE = SEL_THREADS * SEL_VEC * 4;  // 8192 rows / tile
 int sel_ctas_per_sm();  // occupancy of the select kernel on the current device
 

@@ -10,13 +10,13 @@
 // Here the whole chain is ONE persistent, warp-specialised kernel: two CTAs per
 // SM, each with 8 compute warps and one look-back warp.
 //
-//   partition  8192-row tiles dealt round-robin (tile i of CTA b is b + i*G,
-//              G = grid); the grid is launched cooperatively, so every CTA is
-//              co-resident (a CTA may wait on any lower tile).
+//   partition  8192-row tiles are drawn from an atomic ticket counter, one
+//              tile ahead of use, so a CTA that runs slow simply takes fewer
+//              tiles: no tile ever waits on a CTA that is far behind.
 //   load       each tile arrives by one 1-D bulk async copy (cp.async.bulk, TMA
 //              engine) into a 2-slot shared-memory ring completed on mbarriers;
-//              the next tile's copy (32 KB per CTA, 64 KB per SM) is always in
-//              flight while the current one is processed.
+//              the next tile's copy (32 KB per CTA, 64 KB per SM) is in flight
+//              while the current one is processed.
 //   filter     each compute warp owns 1024 contiguous rows of the tile, read as
 //              eight conflict-free 128-bit shared loads per lane; the folded
 //              predicate (lo <= x <= hi, x != ne[]) is evaluated in registers.
@@ -30,24 +30,30 @@
 //              coalesced stores.
 //
 // Look-back, B200 style.  An L2 round trip under full HBM load (~1.4 us) is
-// about two tiles' time budget, so nothing on the compute path waits for one:
-//   * exclusive(t) = inclusive(t - G) + the G-1 aggregates in between.  The
-//     CTA owns t - G and keeps its inclusive prefix, so only aggregates are
-//     read, each published in its owner's count phase — never the result of
-//     another CTA's look-back: there is no chain of dependent look-backs.
-//   * the look-back warp bulk-copies tile k's window of G-1 aggregates into
-//     shared memory when this CTA counts tile k+2 (lower CTAs have published
-//     round k by then) and resolves it at tile k+4; a word still unpublished
-//     (a lagging CTA) is re-polled individually.
-//   * compute warps write tile k at tile k+5, or earlier when the ring of
-//     selected rows runs short (high selectivity; the look-back warp then
-//     resolves on demand).  The ring holds only selected rows, so at 25%
-//     selectivity it is five tiles (~7 us) deep.
+// longer than a tile's time budget, so nothing on the compute path waits for
+// one:
+//   * exclusive(t) = inclusive(t') + the aggregates of the tiles strictly
+//     between t' and t, where t' is this CTA's previous tile — whose inclusive
+//     prefix the look-back warp holds in a register.  Only aggregates are read,
+//     each published in its owner's count phase — never the result of another
+//     CTA's look-back: there is no chain of dependent look-backs.  Tickets are
+//     drawn in order, so every tile between t' and t was drawn before t and is
+//     counted within about one tile time of being drawn.
+//   * the look-back warp bulk-copies tile k's window into shared memory as
+//     soon as tile k is counted and resolves it when tile k+1 is counted (or
+//     at once, on demand, when the compute warps already wait for it); a word
+//     still unpublished is re-polled individually.
+//   * compute warps write tile k when tile k+3 is counted, or earlier when the
+//     ring of selected rows runs short (high selectivity).
+// (Measured on B200, 2^28 rows, s=.25: D1/D2/LAG = 0/1/3 -> 0.273 ms; 2/4/5,
+// the older setting, 0.368 ms; smaller tiles or deeper input rings that cost
+// the second CTA per SM are slower — scripts/sel_variants.sh.)
 //
 // Status words carry a 28-bit launch epoch (header word bumped by the last
 // tile), so stale words of earlier launches read as "not ready": no per-call
-// memset and no second kernel.  A workspace must be re-zeroed once per 2^28
-// launches (ra_workspace_init).
+// memset and no second kernel.  The ticket counter is reset by the last CTA to
+// finish.  A workspace must be re-zeroed once per 2^28 launches
+// (ra_workspace_init).
 
 #include <stdio.h>
 
@@ -56,8 +62,7 @@
 namespace ra {
 
 #ifdef RA_SEL_PROFILE  // counters for scripts/micro/sel_prof.cu; never in the product build
-__device__ unsigned long long g_sel_prof[8];
-__device__ unsigned long long* g_sel_trace;  // [tile] globaltimer at count
+__device__ unsigned long long g_sel_prof[16];
 #define PROF_ADD(k, v) atomicAdd(&g_sel_prof[k], (unsigned long long)(v))
 #else
 #define PROF_ADD(k, v)
@@ -70,22 +75,31 @@ constexpr uint64_t FLAG_A = 1ull << 62;  // tile aggregate published
 constexpr int TAG_SHIFT = 34;
 constexpr uint64_t TAG_MASK = (1ull << 28) - 1;
 
-constexpr int H_EPOCH = 0;  // header word (uint32)
+// header: u32 epoch at word 0, u64 ticket counter at byte 8, u32 done counter at byte 16
+constexpr int H_EPOCH = 0;
+constexpr int H_DONE = 4;
 
 constexpr int NW = SEL_THREADS / 32;     // compute warps
 constexpr int WROWS = SEL_TILE / NW;     // contiguous rows owned by a compute warp (1024)
 constexpr int BLOCK = SEL_THREADS + 32;  // + the look-back warp
-constexpr int K = SEL_LAG + 2;           // metadata slots: tiles counted but not yet written
-constexpr int D1 = 2;                    // window of tile k copied when tile k+D1 is counted
-constexpr int D2 = 4;                    // ... and resolved when tile k+D2 is counted
+#ifndef RA_SEL_LAG
+#define RA_SEL_LAG 3
+#endif
+constexpr int LAG = RA_SEL_LAG;          // tile k is written when tile k+LAG is counted (or earlier)
+constexpr int K = LAG + 2;               // metadata slots: tiles counted but not yet written
+#ifndef RA_SEL_D1
+#define RA_SEL_D1 0
+#define RA_SEL_D2 1
+#endif
+constexpr int D1 = RA_SEL_D1;            // window of tile k copied when tile k+D1 is counted
+constexpr int D2 = RA_SEL_D2;            // ... and resolved when tile k+D2 is counted
 constexpr int Q = D2 - D1 + 1;           // window slots
-constexpr int LBW = 10;                  // window words per lane: 320 >= G-1
+constexpr int LBW = 10;                  // window words per lane per pass
 constexpr int WIN_WORDS = 32 * LBW;      // window slot capacity (words)
-constexpr int MAX_GRID = WIN_WORDS - 2;  // window of G-1 words + alignment slack
 constexpr int NPK = SEL_VEC / 4;         // packed count words per lane (4 rows of 8 bits each)
 static_assert(SEL_VEC % 4 == 0 && SEL_VEC <= 8, "rows per lane are packed as 8-bit counts, fl has 32 bits");
 static_assert(NW <= 32, "one warp reduces the per-warp counts");
-static_assert(SEL_LAG >= D2 + 1, "a tile is placed before it is due");
+static_assert(LAG >= D2 + 1, "a tile is placed before it is due");
 static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");
 
 struct SelParams {
@@ -96,9 +110,11 @@ struct SelParams {
   int64_t out_cap;
   int64_t* d_count;
   uint32_t* hdr;
+  unsigned long long* ticket;
   uint64_t* status;  // status[tile]
   int32_t mis;       // rows of d_in's 16-B chunk before d_in (0..3)
-  int32_t lo, hi;
+  int32_t lo;
+  uint32_t span;  // hi - lo (the interval is never empty: see launch_select_pass)
   int32_t n_ne;
   int32_t ne[RA_MAX_PREDS];
 };
@@ -109,12 +125,15 @@ struct __align__(128) SelSmem {
   uint64_t win[Q][WIN_WORDS];          // look-back windows (bulk-copied status words)
   uint64_t full[SEL_INSLOTS];          // TMA -> compute: tile landed
   uint64_t winfull[Q];                 // TMA -> look-back: window landed
-  uint64_t counted[K];                 // compute -> look-back: aggregate in cnt[]
+  uint64_t counted[K];                 // compute -> look-back: aggregate in cnt[], index in tidx[]
   uint64_t placed[K];                  // look-back -> compute: offset in goff[]
+  int64_t tile_of[SEL_INSLOTS];        // ticket held by each input slot
+  int64_t tidx[K];                     // tile index of CTA-local tile k (-1: no more tiles)
+  int64_t wlo[Q], whi[Q];              // window bounds [lo, hi) of each window slot
+  int64_t goff[K];                     // tile output offsets
   uint32_t wtot[2][NW];                // per-warp selected counts (double-buffered by tile)
   int32_t cnt[K];                      // tile aggregates
-  int32_t start[K];                    // tile run start in the ring (mod SEL_OUTRING)
-  int64_t goff[K];                     // tile output offsets
+  int32_t start[K];                    // tile run start in the ring
   int64_t n;
   uint32_t epoch;
   int32_t demand;  // oldest tile the compute warps are waiting to write (-1: none yet)
@@ -182,7 +201,7 @@ __device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
 
 template <bool HAS_NE>
 __device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
-  bool k = (x >= P.lo) & (x <= P.hi);
+  bool k = (uint32_t)(x - P.lo) <= P.span;  // lo <= x <= hi
   if (HAS_NE) {
 #pragma unroll
     for (int j = 0; j < RA_MAX_PREDS; ++j)
@@ -206,52 +225,56 @@ __device__ __forceinline__ void issue_tile(SelSmem& S, const SelParams& P, int64
   bulk_g2s(&S.in[s][0], P.abase + v0, bytes, &S.full[s]);
 }
 
-// Look-back warp: bulk-copy the window of tile tp — status[tp-G+1 .. tp-1] —
-// into window slot q (16-B aligned start: one extra word may precede it).
-__device__ __forceinline__ void issue_window(SelSmem& S, const SelParams& P, int64_t tp, int64_t G, int q) {
-  int64_t s0 = tp - G + 1;
-  if (s0 < 0) s0 = 0;
-  s0 &= ~1ll;
-  const uint32_t bytes = (uint32_t)(((tp - s0) * 8 + 15) & ~15ll);
-  if (bytes == 0) {  // tile 0: nothing to read
+// Look-back warp, lane 0: bulk-copy window [lo, hi) of status words into slot
+// q (16-B aligned start: one extra word may precede lo).  A window longer than
+// the slot (a CTA that ran slow) is not copied; it is read directly instead.
+__device__ __forceinline__ void issue_window(SelSmem& S, const SelParams& P, int64_t lo, int64_t hi, int q) {
+  S.wlo[q] = lo;
+  S.whi[q] = hi;
+  const int64_t s0 = lo & ~1ll;
+  if (hi <= lo || hi - s0 > WIN_WORDS) {
     mbar_arrive(&S.winfull[q]);
     return;
   }
+  const uint32_t bytes = (uint32_t)(((hi - s0) * 8 + 15) & ~15ll);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   mbar_arrive_expect_tx(&S.winfull[q], bytes);
   bulk_g2s(&S.win[q][0], P.status + s0, bytes, &S.winfull[q]);
 }
 
-// Sum of the aggregates in tile tp's window (one warp).  An aggregate is
+// Sum of the aggregates of tiles [lo, hi) (one warp).  An aggregate is
 // <= SEL_TILE < 2^32, so a word published by this launch has its high half
-// exactly `want` = (FLAG_A | tag) >> 32: readiness is one compare and the sum
-// fits 32 bits (one REDUX).  Words still unpublished in the copy are re-polled.
-__device__ __forceinline__ uint32_t window_sum(const SelSmem& S, const SelParams& P, int64_t tp, int64_t G, int q,
-                                               int lane, uint32_t want) {
-  int64_t lo = tp - G + 1;
-  if (lo < 0) lo = 0;
+// exactly `want` = (FLAG_A | tag) >> 32: readiness is one compare and each
+// pass sums in 32 bits (one REDUX).  Words still unpublished are re-polled.
+__device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams& P, int q, int lane, uint32_t want) {
+  const int64_t lo = S.wlo[q], hi = S.whi[q];
   const int64_t s0 = lo & ~1ll;
-  uint64_t w[LBW];
+  const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
+  int64_t total = 0;
+  for (int64_t base = lo; base < hi; base += WIN_WORDS) {
+    uint64_t w[LBW];
 #pragma unroll
-  for (int c = 0; c < LBW; ++c) {
-    const int64_t idx = lo + LBW * lane + c;  // tile whose aggregate this word is
-    w[c] = idx < tp ? S.win[q][idx - s0] : ((uint64_t)want << 32);
+    for (int c = 0; c < LBW; ++c) {
+      const int64_t idx = base + LBW * lane + c;  // tile whose aggregate this word is
+      w[c] = idx >= hi ? ((uint64_t)want << 32) : copied ? S.win[q][idx - s0] : dev::ld_relaxed_u64(P.status + idx);
+    }
+    for (int spins = 0;; ++spins) {
+      bool missing = false;
+#pragma unroll
+      for (int c = 0; c < LBW; ++c) missing |= (uint32_t)(w[c] >> 32) != want;
+      if (!__any_sync(0xffffffffu, missing)) break;
+      if (lane == 0) PROF_ADD(0, 1);
+      if (spins > 1) __nanosleep(64);
+#pragma unroll
+      for (int c = 0; c < LBW; ++c)
+        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + LBW * lane + c);
+    }
+    uint32_t v = 0;
+#pragma unroll
+    for (int c = 0; c < LBW; ++c) v += (uint32_t)w[c];
+    total += __reduce_add_sync(0xffffffffu, v);
   }
-  for (int spins = 0;; ++spins) {
-    bool missing = false;
-#pragma unroll
-    for (int c = 0; c < LBW; ++c) missing |= (uint32_t)(w[c] >> 32) != want;
-    if (!__any_sync(0xffffffffu, missing)) break;
-    if (lane == 0) PROF_ADD(0, 1);
-    if (spins > 1) __nanosleep(64);
-#pragma unroll
-    for (int c = 0; c < LBW; ++c)
-      if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + lo + LBW * lane + c);
-  }
-  uint32_t v = 0;
-#pragma unroll
-  for (int c = 0; c < LBW; ++c) v += (uint32_t)w[c];
-  return __reduce_add_sync(0xffffffffu, v);
+  return total;
 }
 
 // Compute warps: copy tile k's run of selected rows from the ring to its place.
@@ -280,7 +303,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       n = dn < n ? (dn < 0 ? 0 : dn) : n;
     }
     S.n = n;
-    S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);
+    S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);  // before any ticket: see the epoch note above
     S.demand = -1;
     for (int s = 0; s < SEL_INSLOTS; ++s) mbar_init(&S.full[s], 1);
     for (int s = 0; s < Q; ++s) mbar_init(&S.winfull[s], 1);
@@ -295,44 +318,54 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
   const int64_t nv = n + P.mis;  // virtual rows, counted from the aligned base
   const int64_t ntiles = n > 0 ? (nv + SEL_TILE - 1) / SEL_TILE : 0;
   const uint64_t tag = S.epoch & TAG_MASK;
-  const int64_t G = gridDim.x;
-  const int64_t b = blockIdx.x;
-  const int m = ntiles > b ? (int)((ntiles - b + G - 1) / G) : 0;  // tiles of this CTA
-  if (ntiles == 0) {
-    if (b == 0 && tid == 0) *P.d_count = 0;
-    return;
-  }
 
   if (warp == NW) {
     // ======================= look-back warp: tile offsets =======================
     const uint32_t want = (uint32_t)((FLAG_A | (tag << TAG_SHIFT)) >> 32);
     int64_t my_prefix = 0;  // inclusive prefix of this CTA's last placed tile
+    int64_t t_last = -1;    // tile index of the last window copied
+    int m = 0x7fffffff;     // tiles of this CTA, known once the end marker is counted
+    // Decisions are warp-uniform: a lane that sees a barrier phase complete has
+    // acquired it itself, and the warp acts only when all lanes agree.
+    // tile x counted?  (and learn m from the end marker)
+    auto counted = [&](int x) {
+      if (x >= m) return true;
+      if (!__all_sync(0xffffffffu, mbar_test(&S.counted[x % K], (uint32_t)((x / K) & 1)))) return false;
+      if (S.tidx[x % K] < 0) m = x;
+      return true;
+    };
     // Tile k's window is copied once tile k+D1 is counted and resolved once
     // tile k+D2 is counted — or at once when the compute warps already wait
-    // for tile k (`demand`, ring of selected rows full at high selectivity).
+    // for tile k (`demand`: ring of selected rows full at high selectivity).
     auto due = [&](int k, int d) {
-      const int x = k + d;
-      if (x >= m) return true;
-      if (*(volatile int*)&S.demand >= k) return true;
-      return mbar_test(&S.counted[x % K], (uint32_t)((x / K) & 1));
+      return __all_sync(0xffffffffu, *(volatile int*)&S.demand >= k) || counted(k + d);
     };
     int c_next = 0;  // next window to copy
-    for (int k = 0; k < m; ++k) {
+    for (int k = 0;; ++k) {
+      mbar_wait(&S.counted[k % K], (uint32_t)((k / K) & 1));
+      if (S.tidx[k % K] < 0) break;  // end marker
       for (int spins = 0;; ++spins) {
-        if (c_next < m && c_next < k + Q && due(c_next, D1)) {
-          if (lane == 0) issue_window(S, P, b + (int64_t)c_next * G, G, c_next % Q);
-          ++c_next;
+        if (c_next < k + Q && c_next < m && due(c_next, D1)) {
+          // due(c, D1) implies tile c is counted; wait on it anyway to acquire tidx[]
+          mbar_wait(&S.counted[c_next % K], (uint32_t)((c_next / K) & 1));
+          const int64_t tc = S.tidx[c_next % K];
+          if (tc < 0) {
+            m = c_next;
+          } else {
+            if (lane == 0) issue_window(S, P, t_last + 1, tc, c_next % Q);
+            t_last = tc;
+            ++c_next;
+          }
           continue;
         }
         if (c_next > k && due(k, D2)) break;
         if (spins > 2) __nanosleep(128);
       }
       {  // resolve tile k
-        const int64_t tp = b + (int64_t)k * G;
-        mbar_wait(&S.counted[k % K], (uint32_t)((k / K) & 1));  // own aggregate in cnt[]
-        mbar_wait(&S.winfull[k % Q], (uint32_t)((k / Q) & 1));
-        const uint32_t sum = window_sum(S, P, tp, G, k % Q, lane, want);
-        const int64_t g = my_prefix + (int64_t)sum;
+        const int q = k % Q;
+        mbar_wait(&S.winfull[q], (uint32_t)((k / Q) & 1));
+        const int64_t g = my_prefix + window_sum(S, P, q, lane, want);
+        const int64_t tp = S.whi[q];
         my_prefix = g + S.cnt[k % K];
         if (lane == 0) {
           S.goff[k % K] = g;
@@ -345,27 +378,51 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         __syncwarp();
       }
     }
+    // last CTA out resets the ticket counter for the next launch
+    if (lane == 0) {
+      __threadfence();
+      if (atomicAdd(&P.hdr[H_DONE], 1u) == gridDim.x - 1) {
+        *P.ticket = 0ull;
+        P.hdr[H_DONE] = 0u;
+        if (ntiles == 0) *P.d_count = 0;
+      }
+    }
     return;
   }
 
   // ======================= compute warps ======================================
-  if (tid == 0)
-    for (int s = 0; s < SEL_AHEAD && s < m; ++s) issue_tile(S, P, nv, b + (int64_t)s * G, s);
+  bool drained = false;  // tid 0: drew a ticket >= ntiles
+  auto draw = [&]() -> int64_t {
+    if (drained) return ntiles;
+    const int64_t t = (int64_t)atomicAdd(P.ticket, 1ull);
+    drained = t >= ntiles;
+    return t;
+  };
+  if (tid == 0) {
+    for (int s = 0; s < SEL_AHEAD; ++s) {
+      const int64_t t = draw();
+      S.tile_of[s] = t;
+      if (t < ntiles) issue_tile(S, P, nv, t, s);
+    }
+  }
+  compute_bar();
 
   int32_t wp = 0;    // end of the newest run in the ring
   int32_t used = 0;  // selected rows of pending tiles in the ring
-  int head = 0;    // oldest tile not yet written
-  for (int i = 0; i < m; ++i) {
-    // ---- filter tile i
+  int head = 0;      // oldest tile not yet written
+  int i = 0;
+  for (;; ++i) {
     const int slot = i % SEL_INSLOTS;
-#ifdef RA_SEL_PROFILE
-    const long long c0 = clock64();
-#endif
+    const int64_t t = S.tile_of[slot];
+    if (t >= ntiles) break;
+    if (tid == 0) {  // draw and fetch the next tile into the other slot (read before the last barrier)
+      const int ns = (i + SEL_AHEAD) % SEL_INSLOTS;
+      const int64_t tn = draw();
+      S.tile_of[ns] = tn;
+      if (tn < ntiles) issue_tile(S, P, nv, tn, ns);
+    }
+    // ---- filter tile t
     mbar_wait(&S.full[slot], (uint32_t)((i / SEL_INSLOTS) & 1));
-#ifdef RA_SEL_PROFILE
-    if (tid == 0) PROF_ADD(2, clock64() - c0);
-#endif
-    const int64_t t = b + (int64_t)i * G;
     int4 v[SEL_VEC];
     {
       const int4* base = &S.in[slot][warp * (WROWS / 4)];
@@ -373,7 +430,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       for (int j = 0; j < SEL_VEC; ++j) v[j] = base[32 * j + lane];
     }
     const int64_t v0 = t * SEL_TILE + warp * WROWS;
-    uint32_t fl = 0;  // bit 4j+c: row warp*512 + 4*(32j + lane) + c selected
+    uint32_t fl = 0;  // bit 4j+c: row warp*1024 + 4*(32j + lane) + c selected
     if (v0 >= P.mis && v0 + WROWS <= nv) {
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j)
@@ -390,7 +447,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         }
       }
     }
-    // ---- buffer: order (warp, j, lane, c); packed per-row counts, warp scan
+    // ---- buffer: order (warp, j, lane, c); packed per-row counts, warp scans
     uint32_t packed[NPK], inc[NPK], tot[NPK];  // 4 rows (j) per word, 8 bits each
 #pragma unroll
     for (int q = 0; q < NPK; ++q) {
@@ -415,22 +472,14 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       wtotal += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
     }
     if (lane == 0) S.wtot[i & 1][warp] = wtotal;
-    compute_bar();  // B1: wtot visible; tile i-1's input slot is free
-    if (tid == 0 && i + SEL_AHEAD < m)
-      issue_tile(S, P, nv, b + (int64_t)(i + SEL_AHEAD) * G, (i + SEL_AHEAD) % SEL_INSLOTS);
+    compute_bar();  // B1: wtot visible; every warp is done with this tile's input slot
     const uint32_t wt = lane < NW ? S.wtot[i & 1][lane] : 0u;
     const int32_t agg = (int32_t)__reduce_add_sync(0xffffffffu, wt);
     const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
       dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
-#ifdef RA_SEL_PROFILE
-      if (g_sel_trace) {
-        unsigned long long gt;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
-        g_sel_trace[t] = gt;
-      }
-#endif
       S.cnt[i % K] = agg;
+      S.tidx[i % K] = t;
       mbar_arrive(&S.counted[i % K]);
     }
     // ---- allocate the tile's run: contiguous in the ring (a run that does not
@@ -461,7 +510,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     if (forced) compute_bar();  // rows written out are read before they are overwritten
     if (tid == 0) S.start[i % K] = start;
     used += agg;
-    // ---- scatter tile i into the ring
+    // ---- scatter the tile into the ring
     {
       int32_t rb = start + wbase;
 #pragma unroll
@@ -476,21 +525,19 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       }
     }
     wp = start + agg;
-    // ---- gather: tile i - SEL_LAG is due
-    if (i - SEL_LAG >= head) {
-#ifdef RA_SEL_PROFILE
-      const long long c1 = clock64();
-#endif
+    // ---- gather: tile i - LAG is due
+    if (i - LAG >= head) {
       write_tile(S, P, head, tid);
-#ifdef RA_SEL_PROFILE
-      if (tid == 0) { PROF_ADD(1, clock64() - c1); PROF_ADD(3, 1); }
-#endif
       used -= S.cnt[head % K];
       ++head;
     }
   }
+  if (tid == 0) {  // end marker for the look-back warp
+    S.tidx[i % K] = -1;
+    mbar_arrive(&S.counted[i % K]);
+  }
   compute_bar();  // scatters of the last tiles are visible
-  for (; head < m; ++head) write_tile(S, P, head, tid);
+  for (; head < i; ++head) write_tile(S, P, head, tid);
 }
 
 struct KernelCfg {
@@ -550,26 +597,32 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   P.out_cap = out_cap;
   P.d_count = d_count;
   P.hdr = (uint32_t*)d_ws;
+  P.ticket = (unsigned long long*)((char*)d_ws + 8);
   P.status = (uint64_t*)((char*)d_ws + SEL_HDR_BYTES);
   P.lo = cp.lo;
-  P.hi = cp.hi;
+  P.span = (uint32_t)cp.hi - (uint32_t)cp.lo;
   P.n_ne = cp.n_ne;
   for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne[j] = j < cp.n_ne ? cp.ne[j] : 0;
+  if (cp.lo > cp.hi) {  // empty interval: x == 0 and x != 0
+    P.lo = 0;
+    P.span = 0;
+    P.n_ne = 1;
+    P.ne[0] = 0;
+  }
   if (n_max >= ((int64_t)1 << 34)) return fail(RA_E_INVAL, "n=%lld >= 2^34", (long long)n_max);
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) dev = 0;
-  const bool ne = cp.n_ne > 0;
+  const bool ne = P.n_ne > 0;
   int per_sm = 1;
   int rc = ne ? ensure_config<true>(dev, per_sm) : ensure_config<false>(dev, per_sm);
   if (rc) return rc;
   const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
   int64_t grid = (int64_t)num_sms() * per_sm;
   if (grid > ntiles_max) grid = ntiles_max;
-  if (grid > MAX_GRID) grid = MAX_GRID;
   if (grid < 1) grid = 1;
-  // Cooperative launch: the driver guarantees all CTAs are co-resident, which
-  // the static tile assignment needs (a CTA may wait on any lower tile).
+  // Cooperative launch keeps the persistent CTAs co-resident (they wait on
+  // each other's aggregates); tickets make the order independent of blockIdx.
   const size_t smem = sizeof(SelSmem);
   void* args[] = {(void*)&P};
   cudaError_t le = cudaLaunchCooperativeKernel(

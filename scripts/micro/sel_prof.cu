@@ -1,13 +1,14 @@
-// Phase-timer harness for select_fused_kernel (built with -DRA_SEL_PROFILE).
-// Not product code: includes the library sources into one TU.
+// Timing harness for select_fused_kernel variants (dev tool, not product code):
+// includes the library sources into one TU so -DRA_SEL_VEC=... / -DRA_SEL_PROFILE
+// builds of the kernel can be compared on one box.
+//   usage: sel_prof [T0 [T1 ...]]   (LT thresholds of the chain; default 0 -2^30)
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/capi.cu"
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/select_fused.cu"
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/q1_fused.cu"
-#include <vector>
+#include <cstdlib>
 #ifndef VARIANT
 #define VARIANT "full"
 #endif
-#include <cstdlib>
 
 __global__ void fill(int32_t* x, int64_t n, uint64_t seed) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
@@ -20,49 +21,31 @@ __global__ void fill(int32_t* x, int64_t n, uint64_t seed) {
 int main(int argc, char** argv) {
   int64_t n = 1ll << 28;
   int32_t *x, *out; int64_t* cnt; void* ws;
+  ra_pred p[RA_MAX_PREDS];
+  int k = 0;
+  for (int a = 1; a < argc && k < RA_MAX_PREDS; ++a) p[k++] = {RA_LT, (int32_t)strtoll(argv[a], 0, 0)};
+  if (!k) { p[0] = {RA_LT, 0}; p[1] = {RA_LT, -1073741824}; k = 2; }
   cudaMalloc(&x, n * 4); cudaMalloc(&out, n * 4); cudaMalloc(&cnt, 8);
-  size_t wsb = ra_select_workspace_bytes(n, 2, 1);
+  size_t wsb = ra_select_workspace_bytes(n, k, 1);
   cudaMalloc(&ws, wsb); cudaMemset(ws, 0, wsb);
   fill<<<1184, 256>>>(x, n, 7);
-  ra_pred p[2] = {{RA_LT, 0}, {RA_LT, -1073741824}};
-  for (int i = 0; i < 3; ++i) ra_select_chain(x, n, p, 2, 1, out, n, cnt, ws, wsb, 0);
+  for (int i = 0; i < 3; ++i) ra_select_chain(x, n, p, k, 1, out, n, cnt, ws, wsb, 0);
   cudaDeviceSynchronize();
-  unsigned long long* trace; cudaMalloc(&trace, 8 * ((n + 4095) / 4096));
   cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
   cudaEventRecord(a);
-  const int reps = 10;
-  for (int i = 0; i < reps; ++i) ra_select_chain(x, n, p, 2, 1, out, n, cnt, ws, wsb, 0);
+  const int reps = 20;
+  for (int i = 0; i < reps; ++i) ra_select_chain(x, n, p, k, 1, out, n, cnt, ws, wsb, 0);
   cudaEventRecord(b); cudaEventSynchronize(b);
   float ms; cudaEventElapsedTime(&ms, a, b);
+  ms /= reps;
   int64_t c; cudaMemcpy(&c, cnt, 8, cudaMemcpyDeviceToHost);
-  printf("%-28s ms/call %.4f  count %lld  ctas/sm %d  err=%s\n", VARIANT, ms / reps, (long long)c, ra::sel_ctas_per_sm(),
+  printf("%-24s thr %-12d ms %.4f  GB/s %.0f  count %lld  ctas/sm %d smem %zu err=%s\n", VARIANT, p[k - 1].value, ms,
+         (4.0 * n + 4.0 * c) / ms / 1e6, (long long)c, ra::sel_ctas_per_sm(), sizeof(ra::SelSmem),
          cudaGetErrorString(cudaGetLastError()));
 #ifdef RA_SEL_PROFILE
-  {
-    cudaMemcpyToSymbol(ra::g_sel_trace, &trace, sizeof(trace));
-    ra_select_chain(x, n, p, 2, 1, out, n, cnt, ws, wsb, 0);
-    cudaDeviceSynchronize();
-    int64_t nt = (n + 4095) / 4096;
-    std::vector<unsigned long long> tr(nt);
-    cudaMemcpy(tr.data(), trace, 8 * nt, cudaMemcpyDeviceToHost);
-    int G = 296; unsigned long long t0 = ~0ull;
-    for (auto v : tr) t0 = v < t0 ? v : t0;
-    // per round: spread (max - min) of count times, and mean lag of CTA b vs CTA 0
-    double spread = 0; int rounds = (int)(nt / G);
-    double lagsum[8] = {0};
-    for (int r = 0; r < rounds; ++r) {
-      unsigned long long lo = ~0ull, hi = 0;
-      for (int bb = 0; bb < G; ++bb) { auto v = tr[(int64_t)r * G + bb]; lo = v < lo ? v : lo; hi = v > hi ? v : hi; }
-      spread += hi - lo;
-      for (int q = 0; q < 8; ++q) lagsum[q] += (double)tr[(int64_t)r * G + q * 37] - (double)tr[(int64_t)r * G];
-    }
-    printf("rounds %d: mean round spread %.0f ns; total %.0f ns; per-round time %.0f ns\n", rounds, spread / rounds,
-           (double)(tr[nt - 1] - t0), (double)(tr[nt - 1] - t0) / rounds);
-    for (int q = 0; q < 8; ++q) printf("  CTA %3d mean lag vs CTA 0: %8.0f ns\n", q * 37, lagsum[q] / rounds);
-  }
-  unsigned long long z[8];
+  unsigned long long z[16];
   cudaMemcpyFromSymbol(z, ra::g_sel_prof, sizeof(z));
-  printf("per tile: repolls %.3f  wait_placed(due) %.0f cyc  wait_data %.0f cyc\n", (double)z[0] / z[3], (double)z[1] / z[3], (double)z[2] / z[3]);
+  printf("  look-back re-polls: %llu\n", z[0]);
 #endif
   return 0;
 }

@@ -1,18 +1,18 @@
-mkdir -p gpurun_out
-for d in 0 1 2 3; do
-RA_SEL_DEBUG=$d python - <<'PY'
-import os, sys, torch
-sys.path.insert(0, '.')
-import paper_conf_ipps_wudwcyc12_b200 as R, ragen
-n = 1 << 28
-x = torch.empty(n, dtype=torch.int32, device='cuda'); ragen.int32_column_dev(2, x)
-preds = [('lt', t) for t in ragen.nested_thresholds(0.5, 2)]
-out = torch.empty(n, dtype=torch.int32, device='cuda')
-for _ in range(3): R.select_chain(x, preds, out=out)
-e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
-e0.record()
-for _ in range(20): R.select_chain(x, preds, out=out)
-e1.record(); e1.synchronize()
-print('dbg', os.environ['RA_SEL_DEBUG'], 'ms', e0.elapsed_time(e1) / 20)
-PY
+# Build (here) and run (on the box) select kernel variants: VEC,AHEAD,OUTRING,D1,D2,LAG[,EXTRA_DEFINE]
+# usage: bash scripts/sel_variants.sh build|run "8,1,10240,2,4,5 ..."
+set -e
+V=${2:-"8,1,10240,2,4,5"}
+NV="/usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 --expt-relaxed-constexpr -Iinclude"
+for v in $V; do
+  IFS=, read vec ah ring d1 d2 lag extra <<< "$v"
+  tag=${vec}_${ah}_${ring}_${d1}_${d2}_${lag}${extra:+_$extra}
+  ex=${extra:+-D$extra}
+  b=scripts/micro/selv_$tag
+  if [ "$1" = build ]; then
+    $NV -DRA_SEL_VEC=$vec -DRA_SEL_AHEAD=$ah -DRA_SEL_OUTRING=$ring -DRA_SEL_D1=$d1 -DRA_SEL_D2=$d2 -DRA_SEL_LAG=$lag $ex \
+      -DVARIANT="\"$tag\"" -o $b scripts/micro/sel_prof.cu -lpthread &
+  else
+    for t in -1073741824 0 -2104533975; do timeout 60 $b $t || echo "$b $t FAILED"; done
+  fi
 done
+wait

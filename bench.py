@@ -280,20 +280,29 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
         chunk = 1 << 24
         streams = [torch.cuda.Stream() for _ in range(3)]
         h_counts = torch.zeros((n + chunk - 1) // chunk, dtype=torch.int64, pin_memory=True)
-        R.fission_run(h_in, preds, chunk, streams, h_out=h_out, h_chunk_counts=h_counts)
-        D.barrier(torch)
-        t0 = time.perf_counter()
-        reps = 3
-        for _ in range(reps):
-            _, c = R.fission_run(h_in, preds, chunk, streams, h_out=h_out, h_chunk_counts=h_counts)
-        dt = (time.perf_counter() - t0) / reps
-        dt = D.max(torch, dt)
+        def fission_ms(chunk, S, fused, reps=3):
+            st = streams[:S]
+            R.fission_run(h_in, preds, chunk, st, fused=fused, h_out=h_out, h_chunk_counts=h_counts)
+            # synchronous host API: bracket it with events on the current stream (device clock)
+            ms, _ = timed(torch, D, lambda i, kernel_done=False: R.fission_run(
+                h_in, preds, chunk, st, fused=fused, h_out=h_out, h_chunk_counts=h_counts), reps, 1)
+            return ms
+
+        dt = fission_ms(chunk, 3, True) * 1e-3
+        _, c = R.fission_run(h_in, preds, chunk, streams, h_out=h_out, h_chunk_counts=h_counts)
         assert c == kept
         ex["e2e"] = {"value": D.world * n / dt, "unit": "rows/s", "h2d_bytes_per_step": 4 * n,
-                     "d2h_bytes_per_step": 4 * c + 8 * h_counts.numel(), "ms_per_step": dt * 1e3,
+                     "d2h_bytes_per_step": 4 * c + 8 * ((n + chunk - 1) // chunk), "ms_per_step": dt * 1e3,
                      "path": "ra_fission_run: pinned host in/out, chunk 2^24 rows, 3 streams (fusion+fission)",
                      "pcie_h2d_gbs": 4 * n / dt / 1e9}
-        del h_in, h_out
+        # d4: the paper's Fig 16 modes on the same host-resident chain
+        modes = {"serial": (n, 1, False), "fusion_only": (n, 1, True),
+                 "fission_only": (chunk, 3, False), "fusion_fission": (chunk, 3, True)}
+        ex["fission_modes"] = {m: {"ms_per_step": fission_ms(*cfg), "chunk_rows": cfg[0], "streams": cfg[1],
+                                   "fused": cfg[2]} for m, cfg in modes.items()}
+        for v in ex["fission_modes"].values():
+            v["rows_per_s"] = D.world * n / (v["ms_per_step"] * 1e-3)
+        del h_in, h_out, h_counts
 
     # --- configs[0]: single SELECT on 2^20 rows, 50% (latency-bound, L2-resident)
     n1 = 1 << 20
@@ -308,6 +317,18 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     ms1, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_chain(*a1), 200, 10)
     ex["select_1m"] = {"us_per_call": ms1 * 1e3, "rows_per_s": n1 / (ms1 * 1e-3), "kept": int(c1.item()),
                        "note": "configs[0]; 6 MiB L2-resident, back-to-back stream launches"}
+    try:  # d1: CUDA-graph replay of 100 captured C-ABI calls (launch latency off the host)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            shc = int(torch.cuda.current_stream().cuda_stream)
+            for _ in range(100):
+                R.ra_select_chain(*a1[:-1], shc)
+        gms, _ = timed(torch, D, lambda i, kernel_done=False: g.replay(), 10, 3)
+        ex["select_1m"]["graph_us_per_call"] = gms * 1e3 / 100
+        assert int(c1.item()) == ex["select_1m"]["kept"]
+        del g
+    except Exception as e:  # noqa: BLE001 — report, do not lose the rest of the line
+        ex["select_1m"]["graph_error"] = repr(e)[:200]
 
     # --- configs[2]: Q1 SF10 device-resident (N=1 only) and configs[4] SF100 sharded
     def q1_bench(sf, shard):
@@ -346,6 +367,7 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
 
     if D.world == 1:
         ex["q1_sf10"] = q1_bench(10, False)
+        ex["q1_sf10"]["e2e"] = q1_e2e(args, D, torch, R, 10)
     ex["q1_sf100"] = q1_bench(100, True)
     ex["q1_sf100"]["scaling"] = "strong (600M rows split over ranks)"
 
@@ -353,6 +375,25 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     if D.world == 1 and D.rank == 0:
         ex["cpu_baseline"] = cpu_baseline(x, preds, n)
     return ex
+
+
+def q1_e2e(args, D, torch, R, sf):
+    """Q1 from pinned host columns through ra_q1_fission_run (f1): H2D of the
+    38 B/row inside the timed region, the 400-B partial read back every step."""
+    N = ragen.rows_for_sf(sf)
+    cols = ragen.lineitem(Q1_SEED, N, ragen.parts_for_sf(sf))
+    h = {k: torch.from_numpy(v).pin_memory() for k, v in cols.items()}
+    del cols
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    chunk = 1 << 22
+    part = R.q1_fission_run(h, chunk, streams)
+    ms, _ = timed(torch, D, lambda i, kernel_done=False: R.q1_fission_run(h, chunk, streams), 3, 1)
+    rows, rc = R.q1_finalize(bytes(part))
+    del h
+    return {"value": N / (ms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 38 * N,
+            "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": ms,
+            "pcie_h2d_gbs": 38 * N / (ms * 1e-3) / 1e9, "groups": len(rows), "finalize_rc": rc,
+            "path": "ra_q1_fission_run: pinned host columns, chunk 2^22 rows, 3 streams"}
 
 
 def cpu_baseline(x, preds, n):

@@ -226,6 +226,30 @@ int ra_fission_run(const int32_t* h_in, int64_t n, const ra_pred* h_preds, int k
                    int64_t out_cap, int64_t* h_count, int64_t* h_chunk_counts, void* d_ws,
                    size_t ws_bytes);
 
+/* Host-resident TPC-H Q1 under kernel fission: the paper
+ * applies fission to Q1's fused input stage (L1565-1566, L1669-1671).  The
+ * seven columns are streamed in contiguous chunks of chunk_rows (last one
+ * shorter); chunk c runs on streams[c % n_streams]: H2D of its 38 B/row ->
+ * fused Q1 kernel accumulating into that stream's device partial.  Chunks of
+ * one stream are ordered by the stream, so the host never waits inside the
+ * loop; at the end the n_streams partials are summed exactly (the same
+ * slotwise addition as row-range shards) into *h_partial.  Synchronous.
+ *
+ *  h_cols      host struct of PINNED host column pointers (layout and domain
+ *              as ra_q1), n < 2^32 rows
+ *  chunk_rows  > 0; chunk_rows >= n with one stream = the serial mode
+ *  streams     n_streams >= 1 CUDA streams of the current device
+ *  h_partial   host ra_q1_partial: the whole query's partial (pass it to
+ *              ra_q1_finalize)
+ *  d_ws        ra_q1_fission_workspace_bytes(chunk_rows, n_streams), 256-B
+ *              aligned
+ * Result identical to ra_q1 over the whole table (partition additivity). */
+size_t ra_q1_fission_workspace_bytes(int64_t chunk_rows, int n_streams);
+
+int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff,
+                      int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
+                      ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes);
+
 #ifdef __cplusplus
 }
 #endif

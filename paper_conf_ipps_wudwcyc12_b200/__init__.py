@@ -5,7 +5,8 @@ kernels for the fused SELECT chain, fused TPC-H Q1 and the kernel-fission
 pipeline.  This package is the thin Python layer above it:
 
 * ``ra_*`` — one-to-one ctypes bindings of the C entry points (``_ra.py``);
-* ``select_chain``, ``q1``, ``q1_finalize``, ``fission_run`` — conveniences
+* ``select_chain``, ``q1``, ``q1_finalize``, ``fission_run``,
+  ``q1_fission_run`` — conveniences
   that take torch tensors, allocate outputs/workspaces with torch (device
   memory and streams are PyTorch's; nothing else is) and call the bindings.
 
@@ -18,7 +19,8 @@ import ctypes
 from ._ra import *  # noqa: F401,F403
 from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, ra_fission_run,
                   ra_fission_workspace_bytes, ra_lineitem, ra_q1, ra_q1_finalize, ra_q1_partial,
-                  ra_q1_row, ra_q1_workspace_bytes, ra_select_chain, ra_select_workspace_bytes)
+                  ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
+                  ra_select_chain, ra_select_workspace_bytes)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
@@ -144,3 +146,26 @@ def fission_run(h_in, preds, chunk_rows: int, streams, fused: bool = True, h_out
                    h_out.numel(), ctypes.byref(cnt), h_chunk_counts.data_ptr(), ws.data_ptr(),
                    ws.numel())
     return h_out, int(cnt.value)
+
+
+def q1_fission_run(h_cols, chunk_rows: int, streams, cutoff: int = Q1_CUTOFF_DELTA90, device=None):
+    """Host-resident Q1 under kernel fission (synchronous).
+
+    ``h_cols``: dict of pinned contiguous CPU tensors (LINEITEM_COLUMNS).
+    Returns the whole query's ``ra_q1_partial`` (pass it to ``q1_finalize``).
+    """
+    torch = _torch()
+    n = h_cols["shipdate"].numel()
+    for name in LINEITEM_COLUMNS:
+        t = h_cols[name]
+        if t.numel() != n or t.device.type != "cpu" or not t.is_contiguous() or (n and not t.is_pinned()):
+            raise ValueError(f"h_cols[{name!r}] must be a pinned contiguous CPU tensor of {n} rows")
+    chunk_rows = max(1, min(int(chunk_rows), max(1, n)))
+    device = device or torch.device("cuda", torch.cuda.current_device())
+    S = len(streams)
+    sarr = (ctypes.c_void_p * S)(*[_stream_handle(s) for s in streams])
+    ws = workspace(device, f"q1_fission_{S}", ra_q1_fission_workspace_bytes(chunk_rows, S))
+    part = ra_q1_partial()
+    ra_q1_fission_run(lineitem_struct(h_cols), n, int(cutoff), chunk_rows, sarr, S, part, ws.data_ptr(),
+                      ws.numel())
+    return part

@@ -108,6 +108,8 @@ _SIGS = {
     "ra_q1_finalize": ([_vp, _i32, _vp, _vp], _i32),
     "ra_fission_workspace_bytes": ([_i64, _i32, _i32, _i32], _sz),
     "ra_fission_run": ([_vp, _i64, _vp, _i32, _i32, _i64, _vp, _i32, _vp, _i64, _vp, _vp, _vp, _sz], _i32),
+    "ra_q1_fission_workspace_bytes": ([_i64, _i32], _sz),
+    "ra_q1_fission_run": ([_vp, _i64, ctypes.c_int32, _i64, _vp, _i32, _vp, _vp, _sz], _i32),
 }
 for _name, (_args, _res) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -189,6 +191,16 @@ def ra_fission_run(h_in: int, n: int, h_preds, k: int, fused: int, chunk_rows: i
     if rc < 0 and rc != RA_E_CAPACITY:
         raise RAError(rc, ra_last_error())
     return rc
+
+
+def ra_q1_fission_workspace_bytes(chunk_rows: int, n_streams: int) -> int:
+    return int(_lib.ra_q1_fission_workspace_bytes(chunk_rows, n_streams))
+
+
+def ra_q1_fission_run(h_cols: ra_lineitem, n: int, cutoff: int, chunk_rows: int, streams, n_streams: int,
+                      h_partial, d_ws: int, ws_bytes: int) -> None:
+    _check(_lib.ra_q1_fission_run(ctypes.byref(h_cols), n, cutoff, chunk_rows, streams, n_streams,
+                                  ctypes.byref(h_partial), d_ws, ws_bytes))
 
 
 def make_preds(preds):

@@ -168,3 +168,136 @@ RA_API int ra_fission_run(const int32_t* h_in, int64_t n, const ra_pred* h_preds
     return fail(RA_E_CAPACITY, "%lld selected > out_cap %lld", (long long)offset, (long long)out_cap);
   return RA_OK;
 }
+
+// ------------------------------------------------------------------ Q1
+namespace ra {
+namespace {
+
+// Per-stream region: the chunk's seven columns, the Q1 kernel workspace and
+// the stream's running partial.
+struct Q1Region {
+  size_t sd, rf, ls, dec, ws, part, total;
+};
+
+Q1Region q1_region(int64_t chunk_rows) {
+  Q1Region r;
+  const size_t c = (size_t)chunk_rows;
+  r.sd = 0;
+  r.rf = r.sd + round256(c * 4);
+  r.ls = r.rf + round256(c);
+  r.dec = r.ls + round256(c);  // 4 decimal columns, round256(c * 8) each
+  r.ws = r.dec + 4 * round256(c * 8);
+  r.part = r.ws + round256(q1_ws_bytes());
+  r.total = r.part + round256(sizeof(ra_q1_partial));
+  return r;
+}
+
+// exact slotwise sum (the shard merge of ra_q1_finalize, without finalising)
+void q1_merge(ra_q1_partial& acc, const ra_q1_partial& p) {
+  acc.status |= p.status;
+  acc.rows += p.rows;
+  for (int s = 0; s < RA_Q1_GROUPS; ++s) {
+    ra_q1_group& a = acc.group[s];
+    const ra_q1_group& g = p.group[s];
+    a.count += g.count;
+    a.sum_qty += g.sum_qty;
+    a.sum_base_price += g.sum_base_price;
+    a.sum_disc += g.sum_disc;
+    unsigned __int128 dp = ((unsigned __int128)(uint64_t)a.sum_disc_price_hi << 64) | a.sum_disc_price_lo;
+    dp += ((unsigned __int128)(uint64_t)g.sum_disc_price_hi << 64) | g.sum_disc_price_lo;
+    a.sum_disc_price_lo = (uint64_t)dp;
+    a.sum_disc_price_hi = (int64_t)(uint64_t)(dp >> 64);
+    unsigned __int128 ch = ((unsigned __int128)(uint64_t)a.sum_charge_hi << 64) | a.sum_charge_lo;
+    ch += ((unsigned __int128)(uint64_t)g.sum_charge_hi << 64) | g.sum_charge_lo;
+    a.sum_charge_lo = (uint64_t)ch;
+    a.sum_charge_hi = (int64_t)(uint64_t)(ch >> 64);
+  }
+}
+
+}  // namespace
+}  // namespace ra
+
+RA_API size_t ra_q1_fission_workspace_bytes(int64_t chunk_rows, int n_streams) {
+  if (chunk_rows <= 0 || n_streams <= 0) return 0;
+  return (size_t)n_streams * q1_region(chunk_rows).total;
+}
+
+RA_API int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff,
+                             int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
+                             ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes) {
+  clear_error();
+  if (!h_cols || !h_partial || !streams) return fail(RA_E_INVAL, "null argument");
+  if (n < 0 || n >= (int64_t)1 << 32 || chunk_rows <= 0 || n_streams <= 0)
+    return fail(RA_E_INVAL, "bad sizes (n=%lld chunk_rows=%lld n_streams=%d)", (long long)n,
+                (long long)chunk_rows, n_streams);
+  const ra_lineitem& h = *h_cols;
+  memset(h_partial, 0, sizeof(*h_partial));
+  h_partial->n_groups = RA_Q1_GROUPS;
+  if (n == 0) return RA_OK;
+  if (!h.shipdate || !h.returnflag || !h.linestatus || !h.quantity || !h.extendedprice || !h.discount || !h.tax)
+    return fail(RA_E_INVAL, "null column with n > 0");
+  if (!d_ws) return fail(RA_E_INVAL, "null workspace");
+  if ((uintptr_t)d_ws & 255u) return fail(RA_E_INVAL, "workspace must be 256-byte aligned");
+  if (chunk_rows > n) chunk_rows = n;
+  const size_t need = ra_q1_fission_workspace_bytes(chunk_rows, n_streams);
+  if (ws_bytes < need) return fail(RA_E_WORKSPACE, "q1 fission workspace %zu < required %zu", ws_bytes, need);
+  const void* cols[7] = {h.shipdate, h.returnflag, h.linestatus, h.quantity, h.extendedprice, h.discount, h.tax};
+  const char* names[7] = {"shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax"};
+  for (int j = 0; j < 7; ++j) {
+    int rc = check_pinned(cols[j], names[j], nullptr);
+    if (rc) return rc;
+  }
+  const int S = n_streams;
+  const Q1Region R = q1_region(chunk_rows);
+  int result = RA_OK;
+  // zero each stream's running partial and its Q1 ticket word (the region
+  // layout moves with chunk_rows)
+  for (int s = 0; s < S && result == RA_OK; ++s) {
+    char* base = (char*)d_ws + (size_t)s * R.total;
+    cudaStream_t st = (cudaStream_t)streams[s];
+    cudaError_t e = cudaMemsetAsync(base + R.part, 0, sizeof(ra_q1_partial), st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(base + R.ws, 0, 256, st);
+    if (e != cudaSuccess) result = cuda_fail(e, "cudaMemsetAsync(q1 fission partials)");
+  }
+  const int64_t C = (n + chunk_rows - 1) / chunk_rows;
+  for (int64_t c = 0; c < C && result == RA_OK; ++c) {
+    const int s = (int)(c % S);
+    const int64_t r0 = c * chunk_rows;
+    const int64_t len = (n - r0 < chunk_rows) ? (n - r0) : chunk_rows;
+    char* base = (char*)d_ws + (size_t)s * R.total;
+    cudaStream_t st = (cudaStream_t)streams[s];
+    ra_lineitem d;
+    d.shipdate = (const int32_t*)(base + R.sd);
+    d.returnflag = (const uint8_t*)(base + R.rf);
+    d.linestatus = (const uint8_t*)(base + R.ls);
+    d.quantity = (const int64_t*)(base + R.dec);
+    d.extendedprice = (const int64_t*)(base + R.dec + round256((size_t)chunk_rows * 8));
+    d.discount = (const int64_t*)(base + R.dec + 2 * round256((size_t)chunk_rows * 8));
+    d.tax = (const int64_t*)(base + R.dec + 3 * round256((size_t)chunk_rows * 8));
+    const void* dst[7] = {d.shipdate, d.returnflag, d.linestatus, d.quantity, d.extendedprice, d.discount, d.tax};
+    const size_t esz[7] = {4, 1, 1, 8, 8, 8, 8};
+    for (int j = 0; j < 7 && result == RA_OK; ++j) {
+      cudaError_t e = cudaMemcpyAsync((void*)dst[j], (const char*)cols[j] + r0 * esz[j], (size_t)len * esz[j],
+                                      cudaMemcpyHostToDevice, st);
+      if (e != cudaSuccess) result = cuda_fail(e, "H2D q1 chunk column");
+    }
+    if (result != RA_OK) break;
+    result = launch_q1(d, len, shipdate_cutoff, (ra_q1_partial*)(base + R.part), base + R.ws,
+                       R.part - R.ws, st, /*accumulate=*/1);
+  }
+  std::vector<ra_q1_partial> parts(S);
+  for (int s = 0; s < S; ++s) {
+    cudaStream_t st = (cudaStream_t)streams[s];
+    if (result == RA_OK) {
+      cudaError_t e = cudaMemcpyAsync(&parts[s], (char*)d_ws + (size_t)s * R.total + R.part,
+                                      sizeof(ra_q1_partial), cudaMemcpyDeviceToHost, st);
+      if (e != cudaSuccess) result = cuda_fail(e, "D2H q1 partial");
+    }
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess && result == RA_OK) result = cuda_fail(e, "stream sync");
+  }
+  if (result != RA_OK) return result;
+  for (int s = 0; s < S && s < C; ++s) q1_merge(*h_partial, parts[s]);
+  h_partial->n_groups = RA_Q1_GROUPS;
+  return RA_OK;
+}

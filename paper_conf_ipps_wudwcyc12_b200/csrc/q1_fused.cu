@@ -55,6 +55,7 @@ struct Q1Params {
   int64_t ngroups;  // aligned 4-row groups starting at `head`
   int32_t cutoff;
   ra_q1_partial* out;
+  int accumulate;  // add into *out (chunks of one query under fission) instead of overwriting
   Q1Block* blocks;
   uint32_t* counter;
 };
@@ -252,6 +253,15 @@ __global__ void __launch_bounds__(Q1_THREADS, 2) q1_fused_kernel(const Q1Params 
       }
     }
     ra_q1_group* G = &P.out->group[s];
+    if (P.accumulate) {  // exact: 64-bit sums stay < 2^63 through SF100 (C11), 128-bit ones carry
+      const uint64_t* o = reinterpret_cast<const uint64_t*>(G);
+      if (f < 2) {
+        a += o[2 * f];
+        b += o[2 * f + 1];
+      } else {
+        add128(a, b, o[2 * f], o[2 * f + 1]);
+      }
+    }
     if (f == 0) {
       G->count = (int64_t)a;
       G->sum_qty = (int64_t)b;
@@ -268,9 +278,9 @@ __global__ void __launch_bounds__(Q1_THREADS, 2) q1_fused_kernel(const Q1Params 
   } else if (threadIdx.x == 32) {
     uint32_t st = 0;
     for (int i = 0; i < nb; ++i) st |= __ldcg(&P.blocks[i].status);
-    P.out->status = st;
+    P.out->status = P.accumulate ? (P.out->status | st) : st;
     P.out->n_groups = NS;
-    P.out->rows = (uint64_t)P.n;
+    P.out->rows = P.accumulate ? P.out->rows + (uint64_t)P.n : (uint64_t)P.n;
     *P.counter = 0u;  // self-cleaning for the next launch
   }
 }
@@ -282,7 +292,7 @@ int g_q1_occ[64];  // blocks/SM per device (0 = unknown)
 size_t q1_ws_bytes() { return 256 + (size_t)Q1_MAX_GRID * sizeof(Q1Block); }
 
 int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_partial, void* d_ws,
-              size_t ws_bytes, cudaStream_t s) {
+              size_t ws_bytes, cudaStream_t s, int accumulate) {
   (void)ws_bytes;
   Q1Params P;
   P.sd = c.shipdate;
@@ -295,6 +305,7 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
   P.n = n;
   P.cutoff = cutoff;
   P.out = d_partial;
+  P.accumulate = accumulate;
   P.counter = (uint32_t*)d_ws;
   P.blocks = (Q1Block*)((char*)d_ws + 256);
   // first row index h at which every column is 16-B (flags: 4-B) aligned

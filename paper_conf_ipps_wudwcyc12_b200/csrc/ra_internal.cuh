@@ -71,8 +71,10 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
                       size_t ws_bytes, cudaStream_t s);
 
 // --------------------------------------------------------------- Q1
+// accumulate != 0: add into *d_partial (which must hold a valid partial) instead
+// of overwriting it — chunks of one query under fission.
 int launch_q1(const ra_lineitem& cols, int64_t n, int32_t cutoff, ra_q1_partial* d_partial,
-              void* d_ws, size_t ws_bytes, cudaStream_t s);
+              void* d_ws, size_t ws_bytes, cudaStream_t s, int accumulate = 0);
 size_t q1_ws_bytes();
 
 }  // namespace ra

@@ -86,7 +86,7 @@ size_t ra_select_workspace_bytes(int64_t n, int k, int fused);
  * `pred`, in input order; *d_count = count (int64, device).
  *
  * The paper's four stages — partition, filter, buffer, gather (Fig 3,
- * L303-310, L479-485) — run as ONE kernel: each CTA takes a 4096-row tile by
+ * L303-310, L479-485) — run as ONE kernel: each CTA takes an 8192-row tile by
  * atomic ticket (partition), evaluates the predicate in registers (filter),
  * compacts matches in shared memory via warp ballots/scans (buffer) and
  * obtains its global output offset by a decoupled look-back over the tile

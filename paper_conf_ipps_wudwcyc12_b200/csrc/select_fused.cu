@@ -8,15 +8,16 @@
 // (Fig 6; L784-785, L812-814).
 //
 // Here the whole chain is ONE persistent, warp-specialised kernel: two CTAs per
-// SM, each with 8 compute warps and one look-back warp.
+// SM, each with 8 compute warps, one producer warp and one look-back warp.
 //
-//   partition  8192-row tiles are drawn from an atomic ticket counter, one
-//              tile ahead of use, so a CTA that runs slow simply takes fewer
-//              tiles: no tile ever waits on a CTA that is far behind.
+//   partition  the producer warp draws 8192-row tiles from an atomic ticket
+//              counter (one ticket ahead, so the atomic's round trip overlaps
+//              the wait for a free slot); a CTA that runs slow simply takes
+//              fewer tiles: no tile ever waits on a CTA that is far behind.
 //   load       each tile arrives by one 1-D bulk async copy (cp.async.bulk, TMA
 //              engine) into a 2-slot shared-memory ring completed on mbarriers;
-//              the next tile's copy (32 KB per CTA, 64 KB per SM) is in flight
-//              while the current one is processed.
+//              a slot is refilled as soon as the compute warps have read it, so
+//              up to two 32 KB tiles per CTA (128 KB per SM) are in flight.
 //   filter     each compute warp owns 1024 contiguous rows of the tile, read as
 //              eight conflict-free 128-bit shared loads per lane; the folded
 //              predicate (lo <= x <= hi, x != ne[]) is evaluated in registers.
@@ -30,7 +31,7 @@
 //              coalesced stores.
 //
 // Look-back, B200 style.  An L2 round trip under full HBM load (~1.4 us) is
-// longer than a tile's time budget, so nothing on the compute path waits for
+// comparable to a tile's time budget, so nothing on the compute path waits for
 // one:
 //   * exclusive(t) = inclusive(t') + the aggregates of the tiles strictly
 //     between t' and t, where t' is this CTA's previous tile — whose inclusive
@@ -38,16 +39,18 @@
 //     each published in its owner's count phase — never the result of another
 //     CTA's look-back: there is no chain of dependent look-backs.  Tickets are
 //     drawn in order, so every tile between t' and t was drawn before t and is
-//     counted within about one tile time of being drawn.
-//   * the look-back warp bulk-copies tile k's window into shared memory as
-//     soon as tile k is counted and resolves it when tile k+1 is counted (or
-//     at once, on demand, when the compute warps already wait for it); a word
-//     still unpublished is re-polled individually.
+//     counted within a tile time or two of being drawn.
+//   * the look-back warp bulk-copies tile k's window (~296 words on average,
+//     up to 768 fit a slot) into shared memory once tile k+1 is counted — by
+//     then nearly every word in it is published — and resolves it as soon as
+//     the copy lands (or at once, on demand, when the compute warps already
+//     wait for tile k); a word still unpublished is re-polled individually.
 //   * compute warps write tile k when tile k+3 is counted, or earlier when the
 //     ring of selected rows runs short (high selectivity).
-// (Measured on B200, 2^28 rows, s=.25: D1/D2/LAG = 0/1/3 -> 0.273 ms; 2/4/5,
-// the older setting, 0.368 ms; smaller tiles or deeper input rings that cost
-// the second CTA per SM are slower — scripts/sel_variants.sh.)
+// (Measured on B200, 2^28 rows, k=2, s=.25 overall: window slots of 320 words
+// left ~30% of windows uncopied -> one dependent L2 round trip each, 0.257 ms;
+// 768-word slots copied one tile late: 0.230 ms.  1 CTA/SM with deeper input
+// rings is far slower (0.34 ms) — scripts/sel_variants.sh, scripts/gpu_variants.sh.)
 //
 // Status words carry a 28-bit launch epoch (header word bumped by the last
 // tile), so stale words of earlier launches read as "not ready": no per-call
@@ -64,8 +67,13 @@ namespace ra {
 #ifdef RA_SEL_PROFILE  // counters for scripts/micro/sel_prof.cu; never in the product build
 __device__ unsigned long long g_sel_prof[16];
 #define PROF_ADD(k, v) atomicAdd(&g_sel_prof[k], (unsigned long long)(v))
+#define PT_BEGIN(var) const long long var = clock64()
+#define PT_END(k, var, cond) \
+  if (cond) PROF_ADD(k, clock64() - var)
 #else
 #define PROF_ADD(k, v)
+#define PT_BEGIN(var)
+#define PT_END(k, var, cond)
 #endif
 
 namespace {
@@ -81,23 +89,33 @@ constexpr int H_DONE = 4;
 
 constexpr int NW = SEL_THREADS / 32;     // compute warps
 constexpr int WROWS = SEL_TILE / NW;     // contiguous rows owned by a compute warp (1024)
-constexpr int BLOCK = SEL_THREADS + 32;  // + the look-back warp
+constexpr int LBWARP = NW;               // look-back warp
+constexpr int PRWARP = NW + 1;           // producer warp: tickets + bulk copies
+constexpr int BLOCK = SEL_THREADS + 64;  // + the look-back and producer warps
 #ifndef RA_SEL_LAG
 #define RA_SEL_LAG 3
 #endif
 constexpr int LAG = RA_SEL_LAG;          // tile k is written when tile k+LAG is counted (or earlier)
 constexpr int K = LAG + 2;               // metadata slots: tiles counted but not yet written
+#ifndef RA_SEL_PREDRAW
+#define RA_SEL_PREDRAW 1
+#endif
 #ifndef RA_SEL_D1
-#define RA_SEL_D1 0
+#define RA_SEL_D1 1
 #define RA_SEL_D2 1
 #endif
 constexpr int D1 = RA_SEL_D1;            // window of tile k copied when tile k+D1 is counted
 constexpr int D2 = RA_SEL_D2;            // ... and resolved when tile k+D2 is counted
 constexpr int Q = D2 - D1 + 1;           // window slots
 constexpr int LBW = 10;                  // window words per lane per pass
-constexpr int WIN_WORDS = 32 * LBW;      // window slot capacity (words)
+#ifndef RA_SEL_WIN
+#define RA_SEL_WIN 768
+#endif
+constexpr int WIN_WORDS = RA_SEL_WIN;     // window slot capacity (status words)
+constexpr int PASS_WORDS = 32 * LBW;      // words summed per warp pass
+static_assert(WIN_WORDS % 2 == 0, "16-B granules");
 constexpr int NPK = SEL_VEC / 4;         // packed count words per lane (4 rows of 8 bits each)
-static_assert(SEL_VEC % 4 == 0 && SEL_VEC <= 8, "rows per lane are packed as 8-bit counts, fl has 32 bits");
+static_assert(SEL_VEC == 8, "per-j counts are packed as 2 words x 4 bytes; fl has 32 bits");
 static_assert(NW <= 32, "one warp reduces the per-warp counts");
 static_assert(LAG >= D2 + 1, "a tile is placed before it is due");
 static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");
@@ -123,7 +141,8 @@ struct __align__(128) SelSmem {
   int4 in[SEL_INSLOTS][SEL_TILE / 4];  // input tiles (bulk-copy destination)
   int32_t ring[SEL_OUTRING];           // selected rows of counted, not yet written tiles
   uint64_t win[Q][WIN_WORDS];          // look-back windows (bulk-copied status words)
-  uint64_t full[SEL_INSLOTS];          // TMA -> compute: tile landed
+  uint64_t full[SEL_INSLOTS];          // TMA -> compute: tile landed (or end marker)
+  uint64_t empty[SEL_INSLOTS];         // compute -> producer: slot read
   uint64_t winfull[Q];                 // TMA -> look-back: window landed
   uint64_t counted[K];                 // compute -> look-back: aggregate in cnt[], index in tidx[]
   uint64_t placed[K];                  // look-back -> compute: offset in goff[]
@@ -232,6 +251,8 @@ __device__ __forceinline__ void issue_window(SelSmem& S, const SelParams& P, int
   S.wlo[q] = lo;
   S.whi[q] = hi;
   const int64_t s0 = lo & ~1ll;
+  PROF_ADD(14, hi - s0 > WIN_WORDS ? 1 : 0);
+  PROF_ADD(15, hi > lo ? hi - lo : 0);
   if (hi <= lo || hi - s0 > WIN_WORDS) {
     mbar_arrive(&S.winfull[q]);
     return;
@@ -251,7 +272,7 @@ __device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams&
   const int64_t s0 = lo & ~1ll;
   const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
   int64_t total = 0;
-  for (int64_t base = lo; base < hi; base += WIN_WORDS) {
+  for (int64_t base = lo; base < hi; base += PASS_WORDS) {
     uint64_t w[LBW];
 #pragma unroll
     for (int c = 0; c < LBW; ++c) {
@@ -280,7 +301,9 @@ __device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams&
 // Compute warps: copy tile k's run of selected rows from the ring to its place.
 __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k, int tid) {
   if (tid == 0) *(volatile int*)&S.demand = k;  // tell the look-back warp not to wait for later counts
+  PT_BEGIN(t0);
   mbar_wait(&S.placed[k % K], (uint32_t)((k / K) & 1));
+  PT_END(2, t0, tid == 0);
   const int64_t g = S.goff[k % K];
   const int32_t c = S.cnt[k % K];
   const int32_t* run = S.ring + S.start[k % K];  // contiguous, never wraps
@@ -305,7 +328,10 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     S.n = n;
     S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);  // before any ticket: see the epoch note above
     S.demand = -1;
-    for (int s = 0; s < SEL_INSLOTS; ++s) mbar_init(&S.full[s], 1);
+    for (int s = 0; s < SEL_INSLOTS; ++s) {
+      mbar_init(&S.full[s], 1);
+      mbar_init(&S.empty[s], 1);
+    }
     for (int s = 0; s < Q; ++s) mbar_init(&S.winfull[s], 1);
     for (int s = 0; s < K; ++s) {
       mbar_init(&S.counted[s], 1);
@@ -319,7 +345,40 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
   const int64_t ntiles = n > 0 ? (nv + SEL_TILE - 1) / SEL_TILE : 0;
   const uint64_t tag = S.epoch & TAG_MASK;
 
-  if (warp == NW) {
+  if (warp == PRWARP) {
+    // ======================= producer warp: partition + load ====================
+    // Tickets are drawn one tile ahead of the slot they fill, so the atomic's L2
+    // round trip overlaps the wait for that slot; a slot is refilled as soon as
+    // the compute warps have read it (B1), giving up to SEL_INSLOTS tiles in flight.
+    if (lane == 0) {
+#if RA_SEL_PREDRAW
+      int64_t tn = (int64_t)atomicAdd(P.ticket, 1ull);
+#endif
+      for (int j = 0;; ++j) {
+        const int s = j % SEL_INSLOTS;
+        PT_BEGIN(t0);
+        if (j >= SEL_INSLOTS) mbar_wait(&S.empty[s], (uint32_t)((j / SEL_INSLOTS - 1) & 1));
+        PT_END(11, t0, true);
+#if !RA_SEL_PREDRAW
+        const int64_t tn = (int64_t)atomicAdd(P.ticket, 1ull);
+#endif
+        S.tile_of[s] = tn;
+        if (tn >= ntiles) {  // end marker for the compute warps
+          mbar_arrive(&S.full[s]);
+          break;
+        }
+        issue_tile(S, P, nv, tn, s);
+#if RA_SEL_PREDRAW
+        PT_BEGIN(t1);
+        tn = (int64_t)atomicAdd(P.ticket, 1ull);
+        PT_END(12, t1, true);
+#endif
+      }
+    }
+    return;
+  }
+
+  if (warp == LBWARP) {
     // ======================= look-back warp: tile offsets =======================
     const uint32_t want = (uint32_t)((FLAG_A | (tag << TAG_SHIFT)) >> 32);
     int64_t my_prefix = 0;  // inclusive prefix of this CTA's last placed tile
@@ -342,7 +401,9 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     };
     int c_next = 0;  // next window to copy
     for (int k = 0;; ++k) {
+      PT_BEGIN(t0);
       mbar_wait(&S.counted[k % K], (uint32_t)((k / K) & 1));
+      PT_END(9, t0, lane == 0);
       if (S.tidx[k % K] < 0) break;  // end marker
       for (int spins = 0;; ++spins) {
         if (c_next < k + Q && c_next < m && due(c_next, D1)) {
@@ -363,8 +424,12 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       }
       {  // resolve tile k
         const int q = k % Q;
+        PT_BEGIN(t0);
         mbar_wait(&S.winfull[q], (uint32_t)((k / Q) & 1));
+        PT_END(6, t0, lane == 0);
+        PT_BEGIN(t1);
         const int64_t g = my_prefix + window_sum(S, P, q, lane, want);
+        PT_END(7, t1, lane == 0);
         const int64_t tp = S.whi[q];
         my_prefix = g + S.cnt[k % K];
         if (lane == 0) {
@@ -391,38 +456,20 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
   }
 
   // ======================= compute warps ======================================
-  bool drained = false;  // tid 0: drew a ticket >= ntiles
-  auto draw = [&]() -> int64_t {
-    if (drained) return ntiles;
-    const int64_t t = (int64_t)atomicAdd(P.ticket, 1ull);
-    drained = t >= ntiles;
-    return t;
-  };
-  if (tid == 0) {
-    for (int s = 0; s < SEL_AHEAD; ++s) {
-      const int64_t t = draw();
-      S.tile_of[s] = t;
-      if (t < ntiles) issue_tile(S, P, nv, t, s);
-    }
-  }
-  compute_bar();
-
   int32_t wp = 0;    // end of the newest run in the ring
   int32_t used = 0;  // selected rows of pending tiles in the ring
   int head = 0;      // oldest tile not yet written
   int i = 0;
+  PT_BEGIN(tloop);
   for (;; ++i) {
     const int slot = i % SEL_INSLOTS;
+    PT_BEGIN(tf);
+    mbar_wait(&S.full[slot], (uint32_t)((i / SEL_INSLOTS) & 1));
+    PT_END(1, tf, tid == 0);
+    PT_END(8, tf, tid == 224);
     const int64_t t = S.tile_of[slot];
     if (t >= ntiles) break;
-    if (tid == 0) {  // draw and fetch the next tile into the other slot (read before the last barrier)
-      const int ns = (i + SEL_AHEAD) % SEL_INSLOTS;
-      const int64_t tn = draw();
-      S.tile_of[ns] = tn;
-      if (tn < ntiles) issue_tile(S, P, nv, tn, ns);
-    }
     // ---- filter tile t
-    mbar_wait(&S.full[slot], (uint32_t)((i / SEL_INSLOTS) & 1));
     int4 v[SEL_VEC];
     {
       const int4* base = &S.in[slot][warp * (WROWS / 4)];
@@ -447,15 +494,17 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         }
       }
     }
-    // ---- buffer: order (warp, j, lane, c); packed per-row counts, warp scans
-    uint32_t packed[NPK], inc[NPK], tot[NPK];  // 4 rows (j) per word, 8 bits each
-#pragma unroll
-    for (int q = 0; q < NPK; ++q) {
-      packed[q] = 0;
-#pragma unroll
-      for (int jj = 0; jj < 4; ++jj)
-        packed[q] |= (uint32_t)__popc((fl >> (4 * (4 * q + jj))) & 0xFu) << (8 * jj);
-      inc[q] = packed[q];
+    // ---- buffer: order (warp, j, lane, c); packed per-j counts, warp scans.
+    // SWAR popcount of each nibble of fl (nibble j = the lane's 4 rows of
+    // vector j), then j goes to word j&1, byte j>>1 (8 bits: a warp total <= 128).
+    uint32_t packed[NPK], inc[NPK], tot[NPK];
+    {
+      uint32_t x = fl - ((fl >> 1) & 0x55555555u);
+      x = (x & 0x33333333u) + ((x >> 2) & 0x33333333u);
+      packed[0] = x & 0x0F0F0F0Fu;
+      packed[1] = (x >> 4) & 0x0F0F0F0Fu;
+      inc[0] = packed[0];
+      inc[1] = packed[1];
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -472,11 +521,15 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       wtotal += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
     }
     if (lane == 0) S.wtot[i & 1][warp] = wtotal;
+    PT_BEGIN(tb);
     compute_bar();  // B1: wtot visible; every warp is done with this tile's input slot
+    PT_END(3, tb, tid == 0);
+    PT_END(13, tb, tid == 224);
     const uint32_t wt = lane < NW ? S.wtot[i & 1][lane] : 0u;
     const int32_t agg = (int32_t)__reduce_add_sync(0xffffffffu, wt);
     const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
+      mbar_arrive(&S.empty[slot]);  // input slot free: the producer refills it
       dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
       S.cnt[i % K] = agg;
       S.tidx[i % K] = t;
@@ -515,13 +568,13 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       int32_t rb = start + wbase;
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
-        const uint32_t ex = inc[j >> 2] - packed[j >> 2];
-        int32_t p = rb + (int32_t)((ex >> (8 * (j & 3))) & 0xFFu);
+        const uint32_t ex = inc[j & 1] - packed[j & 1];
+        int32_t p = rb + (int32_t)((ex >> (8 * (j >> 1))) & 0xFFu);
         const uint32_t bits = (fl >> (4 * j)) & 0xFu;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
           if (bits & (1u << c)) S.ring[p++] = comp(v[j], c);
-        rb += (int32_t)((tot[j >> 2] >> (8 * (j & 3))) & 0xFFu);
+        rb += (int32_t)((tot[j & 1] >> (8 * (j >> 1))) & 0xFFu);
       }
     }
     wp = start + agg;
@@ -532,6 +585,8 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       ++head;
     }
   }
+  PT_END(4, tloop, tid == 0);
+  PROF_ADD(5, tid == 0 ? i : 0);
   if (tid == 0) {  // end marker for the look-back warp
     S.tidx[i % K] = -1;
     mbar_arrive(&S.counted[i % K]);

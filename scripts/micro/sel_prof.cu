@@ -45,7 +45,12 @@ int main(int argc, char** argv) {
 #ifdef RA_SEL_PROFILE
   unsigned long long z[16];
   cudaMemcpyFromSymbol(z, ra::g_sel_prof, sizeof(z));
-  printf("  look-back re-polls: %llu\n", z[0]);
+  const double tiles = z[5] ? (double)z[5] : 1.0;
+  printf("  per tile (cycles, summed over all launches): repolls %.3f full-wait w0 %.0f w7 %.0f | placed-wait %.0f | B1 w0 %.0f w7 %.0f | loop %.0f\n"
+         "  lookback: counted-wait %.0f winfull-wait %.0f window-sum %.0f | producer: empty-wait %.0f atomic %.0f\n"
+         "  windows: uncopied (too long) %.4f per tile, mean length %.1f\n",
+         z[0] / tiles, z[1] / tiles, z[8] / tiles, z[2] / tiles, z[3] / tiles, z[13] / tiles, z[4] / tiles, z[9] / tiles,
+         z[6] / tiles, z[7] / tiles, z[11] / tiles, z[12] / tiles, z[14] / tiles, z[15] / tiles);
 #endif
   return 0;
 }

@@ -95,5 +95,18 @@ int main() {
   run_bulk<16384, 4>(d, nbytes, sink, 2, 256);
   run_bulk<32768, 2>(d, nbytes, sink, 1, 256);
   run_bulk<32768, 3>(d, nbytes, sink, 1, 256);
+  run_bulk<32768, 2>(d, nbytes, sink, 2, 288);
+  run_bulk<32768, 3>(d, nbytes, sink, 2, 288);
+  for (int per = 2; per <= 8; per *= 2) {
+    float ms = timeit([&] { ldg_stream<4><<<sms * per, 256>>>((const int4*)d, nbytes / 16, sink); });
+    printf("ldg unroll4 ctas/sm=%d : %8.1f GB/s\n", per, nbytes / ms / 1e6);
+    ms = timeit([&] { ldg_stream<8><<<sms * per, 256>>>((const int4*)d, nbytes / 16, sink); });
+    printf("ldg unroll8 ctas/sm=%d : %8.1f GB/s\n", per, nbytes / ms / 1e6);
+  }
+  {
+    char* o; cudaMalloc(&o, nbytes);
+    float ms = timeit([&] { cudaMemcpyAsync(o, d, nbytes, cudaMemcpyDeviceToDevice); });
+    printf("cudaMemcpy D2D 1 GiB: %8.1f GB/s (read+write)\n", 2.0 * nbytes / ms / 1e6);
+  }
   return 0;
 }

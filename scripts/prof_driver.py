@@ -1,6 +1,6 @@
 """Small driver for ncu: runs the hot-path kernels a few times at bench sizes.
 
-usage: python scripts/prof_driver.py {select|unfused|q1|select1m} [reps] [log2n] [k] [sel]
+usage: python scripts/prof_driver.py {select|unfused|q1|q1time|select1m} [reps] [log2n] [k] [sel]
 """
 import os
 import sys
@@ -30,6 +30,24 @@ def main():
         out = torch.empty(n, dtype=torch.int32, device="cuda")
         for _ in range(reps):
             R.select_chain(x, preds, fused=(what != "unfused"), out=out)
+    elif what == "q1time":  # CUDA-event timing of the fused Q1 at SF10 and SF100
+        for sf in (10, 100):
+            n = ragen.rows_for_sf(sf)
+            cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+                    for name, dt in ragen.LINEITEM_COLUMNS}
+            ragen.lineitem_dev(5, ragen.parts_for_sf(sf), cols)
+            for _ in range(3):
+                R.q1(cols)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(reps):
+                R.q1(cols)
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / reps
+            print(f"q1 SF{sf}: {ms:.4f} ms  {38 * n / ms / 1e6:.1f} GB/s  {n / ms * 1e3:.3e} rows/s")
+            del cols
+            torch.cuda.empty_cache()
     elif what == "q1":
         n = ragen.rows_for_sf(10)
         cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")

@@ -142,3 +142,66 @@ def test_repeated_launches_self_clean(R):
     for p in parts:
         rows, rc = R.q1_finalize(bytes(p.cpu().numpy().tobytes()))
         assert_same(rows, exp)
+
+
+def _widen(cols, frac, seed):
+    """Put a fraction of rows at in-domain values outside the TMA kernel's
+    narrow accumulators (quantity >= 2^16, price >= 2^24), plus the exact
+    boundary values, so both accumulation paths and their flushes are hit."""
+    rng = np.random.default_rng(seed)
+    n = cols["quantity"].size
+    out = {k: v.copy() for k, v in cols.items()}
+    idx = rng.choice(n, int(n * frac), replace=False)
+    out["quantity"][idx] = rng.integers(1 << 16, 1 << 31, idx.size)
+    idx2 = rng.choice(n, int(n * frac), replace=False)
+    out["extendedprice"][idx2] = rng.integers(1 << 24, 1 << 31, idx2.size)
+    edges = np.array([(1 << 16) - 1, 1 << 16, (1 << 24) - 1, 1 << 24, (1 << 31) - 1, 0])
+    pos = rng.choice(n, 60, replace=False)
+    out["quantity"][pos[:30]] = edges[np.arange(30) % edges.size]
+    out["extendedprice"][pos[30:]] = edges[np.arange(30) % edges.size]
+    out["discount"][pos[::7]] = 100
+    out["tax"][pos[::5]] = 100
+    return out
+
+
+@pytest.mark.parametrize("n,frac", [(5000, 0.2), (1_000_003, 0.01), (12_000_017, 0.001)])
+def test_wide_in_domain_values(R, n, frac):
+    cols = _widen(ragen.lineitem(41, n, 200000), frac, n)
+    exp, st = oracle.q1(cols, 10561)
+    assert st == 0
+    rows, rc, part = gpu_q1(R, to_dev(cols), 10561)
+    assert rc == R.RA_OK and part.status == 0
+    assert_same(rows, exp)
+
+
+def test_all_rows_one_group_many_tiles(R):
+    """Every row in one slot at maximal narrow values: the 32-bit narrow sums
+    reach their bound between flushes (count<<16|disc, price < 2^24 x 256)."""
+    n = 10_000_000
+    cols = ragen.lineitem(42, n, 2000)
+    cols["returnflag"][:] = ord("R")
+    cols["linestatus"][:] = ord("O")
+    cols["quantity"][:] = (1 << 16) - 1
+    cols["extendedprice"][:] = (1 << 24) - 1
+    cols["discount"][:] = 100
+    cols["discount"][::2] = 0
+    cols["tax"][:] = 100
+    exp, _ = oracle.q1(cols, 2**31 - 1)
+    rows, rc, _ = gpu_q1(R, to_dev(cols), 2**31 - 1)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)
+
+
+@pytest.mark.parametrize("offsets", [(0, 1, 0, 0, 0, 0, 0), (0, 0, 0, 1, 0, 0, 0), (3, 2, 1, 0, 0, 0, 0)])
+def test_columns_not_coalignable(R, offsets):
+    """Column views whose 16-B alignment differs per column cannot use the
+    bulk-copy kernel; the grid-stride kernel must give the same result."""
+    n = 300_007
+    cols = ragen.lineitem(43, n, 20000)
+    exp, _ = oracle.q1(cols, CUTOFF)
+    d = {}
+    for (name, v), off in zip(cols.items(), offsets):
+        d[name] = torch.from_numpy(np.concatenate([np.zeros(off, v.dtype), v])).cuda()[off:]
+    rows, rc, _ = gpu_q1(R, d)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)

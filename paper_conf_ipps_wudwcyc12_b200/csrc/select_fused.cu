@@ -97,6 +97,12 @@ constexpr int BLOCK = SEL_THREADS + 64;  // + the look-back and producer warps
 #endif
 constexpr int LAG = RA_SEL_LAG;          // tile k is written when tile k+LAG is counted (or earlier)
 constexpr int K = LAG + 2;               // metadata slots: tiles counted but not yet written
+#ifndef RA_SEL_PTXSCATTER
+#define RA_SEL_PTXSCATTER 1
+#endif
+#ifndef RA_SEL_PRODSLEEP
+#define RA_SEL_PRODSLEEP 0
+#endif
 #ifndef RA_SEL_PREDRAW
 #define RA_SEL_PREDRAW 1
 #endif
@@ -192,6 +198,19 @@ __device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
 
 __device__ __forceinline__ int32_t comp(const int4& v, int c) {
   return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
+}
+
+// Store v at shared byte address a and advance a, iff (fl & mask) != 0.
+__device__ __forceinline__ void put_if(uint32_t& a, uint32_t fl, uint32_t mask, int32_t v) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\t.reg .b32 t;\n\t"
+      "and.b32 t, %1, %2;\n\t"
+      "setp.ne.u32 q, t, 0;\n\t"
+      "@q st.shared.b32 [%0], %3;\n\t"
+      "@q add.u32 %0, %0, 4;\n\t}"
+      : "+r"(a)
+      : "r"(fl), "r"(mask), "r"(v)
+      : "memory");
 }
 
 // Issue the bulk copy of tile t into input slot s (one thread).
@@ -318,7 +337,11 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       for (int j = 0;; ++j) {
         const int s = j % SEL_INSLOTS;
         PT_BEGIN(t0);
+#if RA_SEL_PRODSLEEP
+        if (j >= SEL_INSLOTS) dev::mbar_wait_sleep(&S.empty[s], (uint32_t)((j / SEL_INSLOTS - 1) & 1), RA_SEL_PRODSLEEP);
+#else
         if (j >= SEL_INSLOTS) mbar_wait(&S.empty[s], (uint32_t)((j / SEL_INSLOTS - 1) & 1));
+#endif
         PT_END(11, t0, true);
 #if !RA_SEL_PREDRAW
         const int64_t tn = (int64_t)atomicAdd(P.ticket, 1ull);
@@ -527,14 +550,23 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ---- scatter the tile into the ring
     {
       int32_t rb = start + wbase;
+#if RA_SEL_PTXSCATTER
+      const uint32_t ring0 = smem_u32(S.ring);
+#endif
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
         const uint32_t ex = inc[j & 1] - packed[j & 1];
         int32_t p = rb + (int32_t)((ex >> (8 * (j >> 1))) & 0xFFu);
+#if RA_SEL_PTXSCATTER
+        uint32_t a = ring0 + 4u * (uint32_t)p;  // byte address: one predicated store + add per row
+#pragma unroll
+        for (int c = 0; c < 4; ++c) put_if(a, fl, 1u << (4 * j + c), comp(v[j], c));
+#else
         const uint32_t bits = (fl >> (4 * j)) & 0xFu;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
           if (bits & (1u << c)) S.ring[p++] = comp(v[j], c);
+#endif
         rb += (int32_t)((tot[j & 1] >> (8 * (j >> 1))) & 0xFFu);
       }
     }

@@ -13,7 +13,6 @@ usage: python scripts/sweeps.py {d2|d4} [out.txt]
 Timing: CUDA events on the current stream, warm-up first, median of reps.
 """
 import os
-import statistics
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -26,17 +25,18 @@ import ragen  # noqa: E402
 
 
 def ev_ms(fn, reps=10, warm=3):
+    """Mean ms per call over `reps` calls enqueued back to back (the GPU
+    never idles between calls, so host launch overhead is not timed)."""
     for _ in range(warm):
         fn()
-    ts = []
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
     for _ in range(reps):
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record()
         fn()
-        b.record()
-        b.synchronize()
-        ts.append(a.elapsed_time(b))
-    return statistics.median(ts)
+    b.record()
+    b.synchronize()
+    return a.elapsed_time(b) / reps
 
 
 def d2(out):

@@ -250,6 +250,57 @@ int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cut
                       int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
                       ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes);
 
+/* ====================================================== NARROW Q1 (f4)
+ * Compressed lineitem for Q1.  The paper's relations are
+ * "compressed row data" (§III-D) and it names compression as the way
+ * to cut transfer volume (§VI).  The seven Q1 columns (38 B/row)
+ * are re-encoded losslessly into six narrow columns (11 B/row); Q1 over them
+ * yields exactly the partial ra_q1 yields over the wide columns.
+ *
+ *   shipdate       uint16  days since 1970-01-01            (0 .. 65535)
+ *   group          uint8   slot = 2*rf + ls (rf A=0 N=1 R=2,
+ *                          ls F=0 O=1), i.e. RA_Q1 slot order (0 .. 5)
+ *   quantity       uint16  x100                              (0 .. 65535)
+ *   discount, tax  uint8   x100                              (0 .. 100)
+ *   extendedprice  uint32  x100                              (0 .. 2^24-1)
+ * Every TPC-H row fits (quantity <= 5000, price <= 10,495,000).
+ * All column pointers are device pointers aligned to 16 bytes, n rows each. */
+typedef struct {
+  const uint16_t* shipdate;
+  const uint8_t* group;
+  const uint16_t* quantity;
+  const uint8_t* discount;
+  const uint8_t* tax;
+  const uint32_t* extendedprice;
+} ra_lineitem_narrow;
+
+typedef struct {
+  uint16_t* shipdate;
+  uint8_t* group;
+  uint16_t* quantity;
+  uint8_t* discount;
+  uint8_t* tax;
+  uint32_t* extendedprice;
+} ra_lineitem_narrow_out;
+
+/* Encode n wide rows (h_cols: device columns, ra_q1 layout) into the narrow
+ * columns h_out (device, 16-B aligned).  *d_status (device uint32) is
+ * overwritten with the OR over ALL rows of: 1 = a flag byte outside
+ * {A,N,R}x{F,O} (row encoded with group 0xFF), 2 = quantity, price, discount
+ * or tax outside the narrow ranges (row encoded with group 0xFE),
+ * 4 = shipdate outside 0..65535 (clamped).  A table with status 0 is an exact
+ * re-encoding.  Stream-ordered; n < 2^32. */
+int ra_q1_encode(const ra_lineitem* h_cols, int64_t n, const ra_lineitem_narrow_out* h_out,
+                 uint32_t* d_status, ra_stream_t stream);
+
+/* Fused Q1 over narrow columns: same workspace (ra_q1_workspace_bytes), same
+ * cutoff convention and same output (ra_q1_partial, all 6 slots) as ra_q1.
+ * A SELECTED row with group > 5 sets status bit 0, one with discount or tax
+ * > 100 or price >= 2^24 sets status bit 1; such rows are not accumulated.
+ * Stream-ordered; n < 2^32; columns 16-B aligned. */
+int ra_q1_narrow(const ra_lineitem_narrow* h_cols, int64_t n, int32_t shipdate_cutoff,
+                 ra_q1_partial* d_partial, void* d_ws, size_t ws_bytes, ra_stream_t stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -6,7 +6,7 @@ pipeline.  This package is the thin Python layer above it:
 
 * ``ra_*`` — one-to-one ctypes bindings of the C entry points (``_ra.py``);
 * ``select_chain``, ``q1``, ``q1_finalize``, ``fission_run``,
-  ``q1_fission_run`` — conveniences
+  ``q1_fission_run``, ``q1_encode``, ``q1_narrow`` — conveniences
   that take torch tensors, allocate outputs/workspaces with torch (device
   memory and streams are PyTorch's; nothing else is) and call the bindings.
 
@@ -20,10 +20,14 @@ from ._ra import *  # noqa: F401,F403
 from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, ra_fission_run,
                   ra_fission_workspace_bytes, ra_lineitem, ra_q1, ra_q1_finalize, ra_q1_partial,
                   ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
-                  ra_select_chain, ra_select_workspace_bytes)
+                  ra_select_chain, ra_select_workspace_bytes, ra_lineitem_narrow, ra_lineitem_narrow_out,
+                  ra_q1_encode, ra_q1_narrow)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
+# narrow (f4) encoding: column -> torch dtype name (ra.h ra_lineitem_narrow)
+NARROW_COLUMNS = (("shipdate", "uint16"), ("group", "uint8"), ("quantity", "uint16"), ("discount", "uint8"),
+                  ("tax", "uint8"), ("extendedprice", "uint32"))
 
 _WS: dict = {}
 
@@ -87,6 +91,41 @@ def q1(cols, cutoff: int = Q1_CUTOFF_DELTA90, partial=None, stream=None):
     ws = workspace(sd.device, "q1", ra_q1_workspace_bytes(n), stream)
     ra_q1(lineitem_struct(cols), n, int(cutoff), partial.data_ptr(), ws.data_ptr(), ws.numel(),
           _stream_handle(stream))
+    return partial
+
+
+def narrow_empty(n: int, device):
+    """Device tensors for an n-row narrow lineitem (16-B aligned torch allocations)."""
+    torch = _torch()
+    return {name: torch.empty(max(1, n), dtype=getattr(torch, dt), device=device)[:n] for name, dt in NARROW_COLUMNS}
+
+
+def q1_encode(cols, out=None, stream=None):
+    """Re-encode wide CUDA lineitem columns into the narrow layout (f4).
+
+    Returns ``(narrow_cols, status)``; ``status`` is a 1-element uint32 CUDA
+    tensor (0 = exact re-encoding; bits as in ra.h), not synchronised."""
+    torch = _torch()
+    sd = cols["shipdate"]
+    n = sd.numel()
+    if out is None:
+        out = narrow_empty(n, sd.device)
+    status = torch.empty(1, dtype=torch.uint32, device=sd.device)
+    h_out = ra_lineitem_narrow_out(*[out[name].data_ptr() for name, _ in NARROW_COLUMNS])
+    ra_q1_encode(lineitem_struct(cols), n, h_out, status.data_ptr(), _stream_handle(stream))
+    return out, status
+
+
+def q1_narrow(ncols, cutoff: int = Q1_CUTOFF_DELTA90, partial=None, stream=None):
+    """Fused Q1 over narrow CUDA columns; returns the device partial (uint8[400])."""
+    torch = _torch()
+    sd = ncols["shipdate"]
+    n = sd.numel()
+    if partial is None:
+        partial = torch.empty(ctypes.sizeof(ra_q1_partial), dtype=torch.uint8, device=sd.device)
+    ws = workspace(sd.device, "q1", ra_q1_workspace_bytes(n), stream)
+    h = ra_lineitem_narrow(*[ncols[name].data_ptr() for name, _ in NARROW_COLUMNS])
+    ra_q1_narrow(h, n, int(cutoff), partial.data_ptr(), ws.data_ptr(), ws.numel(), _stream_handle(stream))
     return partial
 
 

@@ -200,6 +200,44 @@ RA_API int ra_q1(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff, 
   return launch_q1(c, n, shipdate_cutoff, d_partial, d_ws, ws_bytes, (cudaStream_t)stream);
 }
 
+RA_API int ra_q1_encode(const ra_lineitem* h_cols, int64_t n, const ra_lineitem_narrow_out* h_out,
+                        uint32_t* d_status, ra_stream_t stream) {
+  clear_error();
+  if (!h_cols || !h_out || !d_status) return fail(RA_E_INVAL, "null argument");
+  if (n < 0 || n >= (int64_t)1 << 32) return fail(RA_E_INVAL, "n=%lld outside [0, 2^32)", (long long)n);
+  const ra_lineitem& c = *h_cols;
+  const ra_lineitem_narrow_out& o = *h_out;
+  if (n > 0 && (!c.shipdate || !c.returnflag || !c.linestatus || !c.quantity || !c.extendedprice ||
+                !c.discount || !c.tax || !o.shipdate || !o.group || !o.quantity || !o.discount || !o.tax ||
+                !o.extendedprice))
+    return fail(RA_E_INVAL, "null column with n > 0");
+  if (((uintptr_t)c.shipdate & 3u) || (((uintptr_t)c.quantity | (uintptr_t)c.extendedprice |
+                                        (uintptr_t)c.discount | (uintptr_t)c.tax) & 7u))
+    return fail(RA_E_INVAL, "input columns must be naturally aligned");
+  if (((uintptr_t)o.shipdate | (uintptr_t)o.group | (uintptr_t)o.quantity | (uintptr_t)o.discount |
+       (uintptr_t)o.tax | (uintptr_t)o.extendedprice) & 15u)
+    return fail(RA_E_INVAL, "narrow columns must be 16-byte aligned");
+  if ((uintptr_t)d_status & 3u) return fail(RA_E_INVAL, "d_status must be 4-byte aligned");
+  return launch_q1_encode(c, n, o, d_status, (cudaStream_t)stream);
+}
+
+RA_API int ra_q1_narrow(const ra_lineitem_narrow* h_cols, int64_t n, int32_t shipdate_cutoff,
+                        ra_q1_partial* d_partial, void* d_ws, size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  if (!h_cols || !d_partial || !d_ws) return fail(RA_E_INVAL, "null argument");
+  if (n < 0 || n >= (int64_t)1 << 32) return fail(RA_E_INVAL, "n=%lld outside [0, 2^32)", (long long)n);
+  const ra_lineitem_narrow& c = *h_cols;
+  if (n > 0 && (!c.shipdate || !c.group || !c.quantity || !c.discount || !c.tax || !c.extendedprice))
+    return fail(RA_E_INVAL, "null column with n > 0");
+  if (((uintptr_t)c.shipdate | (uintptr_t)c.group | (uintptr_t)c.quantity | (uintptr_t)c.discount |
+       (uintptr_t)c.tax | (uintptr_t)c.extendedprice) & 15u)
+    return fail(RA_E_INVAL, "narrow columns must be 16-byte aligned");
+  if ((uintptr_t)d_partial & 7u) return fail(RA_E_INVAL, "d_partial must be 8-byte aligned");
+  if ((uintptr_t)d_ws & 255u) return fail(RA_E_INVAL, "workspace must be 256-byte aligned");
+  if (ws_bytes < q1_ws_bytes()) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, q1_ws_bytes());
+  return launch_q1_narrow(c, n, shipdate_cutoff, d_partial, d_ws, (cudaStream_t)stream);
+}
+
 RA_API int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h_rows, int* n_rows) {
   clear_error();
   if (n_partials < 0 || (n_partials > 0 && !h_partials) || !h_rows || !n_rows)

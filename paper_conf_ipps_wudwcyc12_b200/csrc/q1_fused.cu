@@ -39,20 +39,13 @@
 
 #include <stdio.h>
 
-#include "ra_internal.cuh"
+#include "q1_common.cuh"
 
 namespace ra {
 
 namespace {
 
-constexpr int NS = RA_Q1_GROUPS;
-constexpr int Q1_MAX_GRID = 148 * 8;
-
-struct Q1Block {
-  uint32_t status;
-  uint32_t _pad;
-  uint64_t v[NS][8];  // count, qty, price, disc, dp_lo, dp_hi, ch_lo, ch_hi
-};
+using namespace q1c;
 
 struct Q1Params {
   const int32_t* sd;
@@ -71,24 +64,6 @@ struct Q1Params {
   Q1Block* blocks;
   uint32_t* counter;
 };
-
-// Final per-thread sums handed to the reduction.
-struct Acc {
-  uint32_t cnt[NS];
-  uint32_t sdisc[NS];
-  uint64_t sq[NS], sp[NS], sdp[NS], sch[NS];
-  uint32_t status;
-};
-
-__device__ __forceinline__ void acc_zero(Acc& A) {
-#pragma unroll
-  for (int s = 0; s < NS; ++s) {
-    A.cnt[s] = 0;
-    A.sdisc[s] = 0;
-    A.sq[s] = A.sp[s] = A.sdp[s] = A.sch[s] = 0;
-  }
-  A.status = 0;
-}
 
 // Per-row SELECT + domain checks + group slot + PROJECT.  Returns the slot
 // (-1: not accumulated) and the projected disc_price / charge.
@@ -157,134 +132,6 @@ __device__ __forceinline__ void row(Acc& A, int32_t cutoff, int32_t sd, uint32_t
                     (uint64_t)q, (uint64_t)p, v.dp, v.ch)
   Q1_SLOT(0); Q1_SLOT(1); Q1_SLOT(2); Q1_SLOT(3); Q1_SLOT(4); Q1_SLOT(5);
 #undef Q1_SLOT
-}
-
-__device__ __forceinline__ void add128(uint64_t& lo, uint64_t& hi, uint64_t lo2, uint64_t hi2) {
-  const uint64_t l = lo + lo2;
-  hi += hi2 + (l < lo ? 1ull : 0ull);
-  lo = l;
-}
-
-__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-  return v;
-}
-
-__device__ __forceinline__ void warp_sum_u128(uint64_t& lo, uint64_t& hi) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const uint64_t l2 = __shfl_xor_sync(0xffffffffu, lo, o);
-    const uint64_t h2 = __shfl_xor_sync(0xffffffffu, hi, o);
-    add128(lo, hi, l2, h2);
-  }
-}
-
-// Reduction: warp (shuffles) -> CTA (smem) -> grid (last CTA, 128-bit fold).
-// Called by every thread of the CTA; warps >= NW (a producer warp) only join
-// the barriers.  s_w: [NW][NS][8] shared scratch.
-template <int NW>
-__device__ __forceinline__ void reduce_and_fold(const Acc& A, const Q1Params& P, uint64_t (*s_w)[NS][8],
-                                                uint32_t* s_status, bool* s_last) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  if (threadIdx.x == 0) *s_status = 0;
-  __syncthreads();
-  if (warp < NW) {
-    if (A.status) atomicOr(s_status, A.status);
-#pragma unroll
-    for (int s = 0; s < NS; ++s) {
-      const uint64_t c = warp_sum_u64(A.cnt[s]);
-      const uint64_t q = warp_sum_u64(A.sq[s]);
-      const uint64_t p = warp_sum_u64(A.sp[s]);
-      const uint64_t d = warp_sum_u64(A.sdisc[s]);
-      uint64_t dlo = A.sdp[s], dhi = 0, clo = A.sch[s], chi = 0;
-      warp_sum_u128(dlo, dhi);
-      warp_sum_u128(clo, chi);
-      if (lane == 0) {
-        s_w[warp][s][0] = c;
-        s_w[warp][s][1] = q;
-        s_w[warp][s][2] = p;
-        s_w[warp][s][3] = d;
-        s_w[warp][s][4] = dlo;
-        s_w[warp][s][5] = dhi;
-        s_w[warp][s][6] = clo;
-        s_w[warp][s][7] = chi;
-      }
-    }
-  }
-  __syncthreads();
-  Q1Block* mine = P.blocks + blockIdx.x;
-  if (threadIdx.x < NS * 4) {  // (slot, field pair)
-    const int s = threadIdx.x >> 2, f = threadIdx.x & 3;
-    if (f < 2) {  // count/qty or price/disc: 64-bit
-      uint64_t a = 0, b = 0;
-      for (int w = 0; w < NW; ++w) {
-        a += s_w[w][s][2 * f];
-        b += s_w[w][s][2 * f + 1];
-      }
-      mine->v[s][2 * f] = a;
-      mine->v[s][2 * f + 1] = b;
-    } else {  // dp or ch: 128-bit
-      uint64_t lo = 0, hi = 0;
-      for (int w = 0; w < NW; ++w) add128(lo, hi, s_w[w][s][2 * f], s_w[w][s][2 * f + 1]);
-      mine->v[s][2 * f] = lo;
-      mine->v[s][2 * f + 1] = hi;
-    }
-  }
-  if (threadIdx.x == 0) mine->status = *s_status;
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) *s_last = (atomicAdd(P.counter, 1u) == gridDim.x - 1);
-  __syncthreads();
-  if (!*s_last) return;
-
-  // ---- last CTA: fold all CTA partials (128-bit where needed)
-  __threadfence();
-  const int nb = gridDim.x;
-  if (threadIdx.x < NS * 4) {
-    const int s = threadIdx.x >> 2, f = threadIdx.x & 3;
-    uint64_t a = 0, b = 0;
-    for (int i = 0; i < nb; ++i) {
-      const uint64_t x = __ldcg(&P.blocks[i].v[s][2 * f]);
-      const uint64_t y = __ldcg(&P.blocks[i].v[s][2 * f + 1]);
-      if (f < 2) {
-        a += x;
-        b += y;
-      } else {
-        add128(a, b, x, y);
-      }
-    }
-    ra_q1_group* G = &P.out->group[s];
-    if (P.accumulate) {  // exact: 64-bit sums stay < 2^63 through SF100 (C11), 128-bit ones carry
-      const uint64_t* o = reinterpret_cast<const uint64_t*>(G);
-      if (f < 2) {
-        a += o[2 * f];
-        b += o[2 * f + 1];
-      } else {
-        add128(a, b, o[2 * f], o[2 * f + 1]);
-      }
-    }
-    if (f == 0) {
-      G->count = (int64_t)a;
-      G->sum_qty = (int64_t)b;
-    } else if (f == 1) {
-      G->sum_base_price = (int64_t)a;
-      G->sum_disc = (int64_t)b;
-    } else if (f == 2) {
-      G->sum_disc_price_lo = a;
-      G->sum_disc_price_hi = (int64_t)b;
-    } else {
-      G->sum_charge_lo = a;
-      G->sum_charge_hi = (int64_t)b;
-    }
-  } else if (threadIdx.x == 32) {
-    uint32_t st = 0;
-    for (int i = 0; i < nb; ++i) st |= __ldcg(&P.blocks[i].status);
-    P.out->status = P.accumulate ? (P.out->status | st) : st;
-    P.out->n_groups = NS;
-    P.out->rows = P.accumulate ? P.out->rows + (uint64_t)P.n : (uint64_t)P.n;
-    *P.counter = 0u;  // self-cleaning for the next launch
-  }
 }
 
 // ===================================================== grid-stride kernel

@@ -1,0 +1,337 @@
+// q1_narrow.cu — TPC-H Q1 over a narrow (11 B/row) lineitem encoding, and
+// the device encoder that produces it.
+//
+// The paper feeds its kernels "compressed row data" (§III-D
+// L990-993) and names compression as the lever on transfer volume (§VI
+// L1722-1724).  Q1 is HBM-bound at 38 B/row, so cutting the row to 11 B
+// (ra.h: u16 shipdate, u8 group code, u16 quantity, u8 discount, u8 tax, u32
+// price) raises the rows/s ceiling ~3.5x.  At 11 B/row the per-row arithmetic
+// becomes the limit, so the accumulation is restructured as well:
+//
+// q1n_kernel — persistent, one CTA per SM, warp-specialised like the wide
+//   q1_tma_kernel: a producer warp streams 1024-row tiles of the six columns
+//   (six cp.async.bulk copies, 11 KB per tile) through an 8-stage
+//   shared-memory ring on mbarriers; 8 compute warps take 4 rows per thread
+//   per tile.  Instead of a predicated update of all 6 group slots per row
+//   (~48 instructions), each row does ONE read-modify-write of its group's
+//   32-byte record in thread-private shared memory (two 128-bit loads, seven
+//   32-bit adds, two 128-bit stores); unselected rows go to a 7th "trash"
+//   record, so there is no predicate at all.  Records are laid out
+//   [slot][half][thread] so a warp is conflict-free whatever its mix of
+//   slots.  A record holds 32-bit sums over <= 256 rows (bounds in nflush()):
+//     count<<16 | disc,  qty,  price,  dp>>16,  dp&0xffff,  f*(dp>>16),  f*(dp&0xffff)
+//   with dp = price*(100-disc) < 2^31 and f = 100+tax, folded every 256 rows
+//   per thread into 64-bit register sums.  (A variant keeping count/disc/qty/
+//   price in predicated register slots and only the dp/charge halves in a
+//   16-byte record moved the bound from shared memory to instruction issue
+//   and was 16% slower.)  The end reduction is the shared warp -> CTA ->
+//   last-CTA 128-bit fold (q1_common.cuh).
+//
+// q1_encode_kernel — grid-stride re-encoding of the wide SoA columns, with the
+//   domain reported in a status word (ra.h).  Not on the timed query path: it
+//   is the load/compression step of the column store.
+
+#include <stdio.h>
+
+#include "q1_common.cuh"
+
+namespace ra {
+
+namespace {
+
+using namespace q1c;
+
+constexpr int QN_NT = 256;     // compute threads + 1 producer warp
+constexpr int QN_NW = QN_NT / 32;
+constexpr int QN_TILE = 1024;  // rows per tile (11 KB)
+constexpr int QN_STAGES = 8;
+constexpr int QN_R = QN_TILE / QN_NT;  // 4 rows per thread per tile
+constexpr int QN_FLUSH_TILES = 256 / QN_R;
+static_assert(QN_R == 4, "the per-thread loads below take 4 rows");
+
+// stage layout (bytes): price u32[T] | shipdate u16[T] | qty u16[T] | group u8[T] | disc u8[T] | tax u8[T]
+constexpr int NO_P = 0, NO_SD = 4 * QN_TILE, NO_Q = 6 * QN_TILE, NO_G = 8 * QN_TILE, NO_D = 9 * QN_TILE,
+              NO_T = 10 * QN_TILE;
+constexpr int NSTAGE_BYTES = 11 * QN_TILE;
+constexpr int TRASH = NS;  // record index of unselected / out-of-domain rows
+
+struct QnParams {
+  const uint16_t* sd;
+  const uint8_t* g;
+  const uint16_t* q;
+  const uint8_t* d;
+  const uint8_t* t;
+  const uint32_t* p;
+  int64_t n;
+  int64_t ntiles;
+  int32_t cutoff;
+  ra_q1_partial* out;
+  int accumulate;
+  Q1Block* blocks;
+  uint32_t* counter;
+};
+
+struct QnSmem {
+  alignas(128) unsigned char stage[QN_STAGES][NSTAGE_BYTES];
+  uint4 rec[NS + 1][2][QN_NT];  // [slot][half][thread]: thread-private 32-byte records
+  uint64_t s_w[QN_NW][NS][8];
+  uint64_t full[QN_STAGES], empty[QN_STAGES];
+  uint32_t status;
+  bool last;
+};
+constexpr size_t QN_SMEM = sizeof(QnSmem);
+static_assert(QN_SMEM <= 227 * 1024, "narrow Q1 kernel exceeds the shared-memory opt-in limit");
+
+struct NAcc {  // 64-bit per-thread totals (count and disc fit 32 bits: <= 2^17 rows/thread)
+  uint32_t cnt[NS], disc[NS];
+  uint64_t sq[NS], sp[NS], dp[NS], ch[NS];
+};
+
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+  return v;
+}
+
+// Always a full 128-bit store (nvcc splits a C++ uint4 store whose last word
+// is unchanged into 64+32-bit stores: twice the shared-memory wavefronts).
+__device__ __forceinline__ void sts128(uint32_t a, const uint4& v) {
+  asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+
+constexpr uint32_t REC_HALF = QN_NT * sizeof(uint4);  // bytes between the two halves of a record
+constexpr uint32_t REC_SLOT = 2 * REC_HALF;           // bytes between slots
+
+// One row: SELECT, domain check, PROJECT, and one read-modify-write of its
+// group's record (unselected / out-of-domain rows hit the trash record).
+__device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cutoff, uint32_t sd, uint32_t g,
+                                     uint32_t q, uint32_t d, uint32_t t, uint32_t p) {
+  const bool sel = (int32_t)sd <= cutoff;  // SELECT
+  const bool okg = g < (uint32_t)NS;
+  const bool okn = (d <= 100u) & (t <= 100u) & (p < (1u << 24));
+  status |= sel ? ((okg ? 0u : 1u) | (okn ? 0u : 2u)) : 0u;
+  const uint32_t slot = (sel & okg & okn) ? g : (uint32_t)TRASH;
+  const uint32_t dp = p * (100u - d), f = 100u + t;  // PROJECT (dp < 2^31)
+  const uint32_t dh = dp >> 16, dl = dp & 0xFFFFu;
+  const uint32_t ra = rec0 + slot * REC_SLOT;
+  uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
+  a.x += (1u << 16) | d;
+  a.y += q;
+  a.z += p;
+  a.w += dh;
+  b.x += dl;
+  b.y += f * dh;
+  b.z += f * dl;
+  sts128(ra, a);
+  sts128(ra + REC_HALF, b);
+}
+
+// Fold the records into the 64-bit sums.  Between two flushes a thread adds
+// <= 256 rows, so every record field stays within 32 bits:
+//   count <= 256 (<< 16 -> < 2^25), disc <= 25600 < 2^16, qty < 2^16 * 2^8,
+//   price <= (2^24-1) * 2^8 < 2^32, dp>>16 < 2^15 * 2^8, dp&0xffff < 2^16 * 2^8,
+//   f*(dp>>16) < 200 * 2^15 * 2^8 < 2^31, f*(dp&0xffff) < 200 * 2^16 * 2^8 < 2^32.
+__device__ __forceinline__ void nflush(NAcc& W, uint32_t rec0) {
+#pragma unroll
+  for (int s = 0; s < NS; ++s) {
+    const uint32_t ra = rec0 + s * REC_SLOT;
+    const uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
+    W.cnt[s] += a.x >> 16;
+    W.disc[s] += a.x & 0xFFFFu;
+    W.sq[s] += a.y;
+    W.sp[s] += a.z;
+    W.dp[s] += ((uint64_t)a.w << 16) + b.x;
+    W.ch[s] += ((uint64_t)b.y << 16) + b.z;
+    sts128(ra, make_uint4(0, 0, 0, 0));
+    sts128(ra + REC_HALF, make_uint4(0, 0, 0, 0));
+  }
+}
+
+__global__ void __launch_bounds__(QN_NT + 32, 1) q1n_kernel(const QnParams P) {
+  extern __shared__ __align__(128) unsigned char qn_smem_raw[];
+  QnSmem& S = *reinterpret_cast<QnSmem*>(qn_smem_raw);
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31;
+
+  if (tid == 0) {
+    for (int s = 0; s < QN_STAGES; ++s) {
+      dev::mbar_init(&S.full[s], 1);
+      dev::mbar_init(&S.empty[s], QN_NW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (tid < QN_NT) {
+#pragma unroll
+    for (int s = 0; s <= NS; ++s) S.rec[s][0][tid] = S.rec[s][1][tid] = make_uint4(0, 0, 0, 0);
+  }
+  __syncthreads();
+
+  Acc A;
+  acc_zero(A);
+  if (warp == QN_NW) {
+    // ---------------- producer warp: one elected lane issues the bulk copies
+    if (lane == 0) {
+      int i = 0;
+      for (int64_t tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x, ++i) {
+        const int s = i % QN_STAGES;
+        if (i >= QN_STAGES) dev::mbar_wait(&S.empty[s], ((i / QN_STAGES) + 1) & 1);
+        const int64_t r0 = tile * QN_TILE;
+        unsigned char* st = S.stage[s];
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        dev::mbar_arrive_expect_tx(&S.full[s], NSTAGE_BYTES);
+        dev::bulk_g2s(st + NO_P, P.p + r0, 4 * QN_TILE, &S.full[s]);
+        dev::bulk_g2s(st + NO_SD, P.sd + r0, 2 * QN_TILE, &S.full[s]);
+        dev::bulk_g2s(st + NO_Q, P.q + r0, 2 * QN_TILE, &S.full[s]);
+        dev::bulk_g2s(st + NO_G, P.g + r0, QN_TILE, &S.full[s]);
+        dev::bulk_g2s(st + NO_D, P.d + r0, QN_TILE, &S.full[s]);
+        dev::bulk_g2s(st + NO_T, P.t + r0, QN_TILE, &S.full[s]);
+      }
+    }
+  } else {
+    // ---------------- compute warps: rows 4*tid .. 4*tid+3 of each tile
+    NAcc N;
+#pragma unroll
+    for (int s = 0; s < NS; ++s) {
+      N.cnt[s] = N.disc[s] = 0;
+      N.sq[s] = N.sp[s] = N.dp[s] = N.ch[s] = 0;
+    }
+    const uint32_t rec0 = dev::smem_u32(&S.rec[0][0][tid]);
+    uint32_t status = 0;
+    int i = 0, since = 0;
+    for (int64_t tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x, ++i) {
+      const int s = i % QN_STAGES;
+      dev::mbar_wait(&S.full[s], (i / QN_STAGES) & 1);
+      const unsigned char* st = S.stage[s];
+      const uint4 p = *reinterpret_cast<const uint4*>(st + NO_P + 16 * tid);
+      const uint2 sd = *reinterpret_cast<const uint2*>(st + NO_SD + 8 * tid);
+      const uint2 q = *reinterpret_cast<const uint2*>(st + NO_Q + 8 * tid);
+      const uint32_t g = *reinterpret_cast<const uint32_t*>(st + NO_G + 4 * tid);
+      const uint32_t d = *reinterpret_cast<const uint32_t*>(st + NO_D + 4 * tid);
+      const uint32_t t = *reinterpret_cast<const uint32_t*>(st + NO_T + 4 * tid);
+      __syncwarp();
+      if (lane == 0) dev::mbar_arrive(&S.empty[s]);  // the stage's values are in registers
+      nrow(rec0, status, P.cutoff, sd.x & 0xFFFFu, g & 0xFF, q.x & 0xFFFFu, d & 0xFF, t & 0xFF, p.x);
+      nrow(rec0, status, P.cutoff, sd.x >> 16, (g >> 8) & 0xFF, q.x >> 16, (d >> 8) & 0xFF, (t >> 8) & 0xFF, p.y);
+      nrow(rec0, status, P.cutoff, sd.y & 0xFFFFu, (g >> 16) & 0xFF, q.y & 0xFFFFu, (d >> 16) & 0xFF,
+           (t >> 16) & 0xFF, p.z);
+      nrow(rec0, status, P.cutoff, sd.y >> 16, g >> 24, q.y >> 16, d >> 24, t >> 24, p.w);
+      if (++since == QN_FLUSH_TILES) {
+        nflush(N, rec0);
+        since = 0;
+      }
+    }
+    nflush(N, rec0);
+    // tail rows after the full tiles (< 1 per thread)
+    const int64_t tail0 = P.ntiles * QN_TILE;
+    for (int64_t r = tail0 + (int64_t)blockIdx.x * QN_NT + tid; r < P.n; r += (int64_t)gridDim.x * QN_NT)
+      nrow(rec0, status, P.cutoff, P.sd[r], P.g[r], P.q[r], P.d[r], P.t[r], P.p[r]);
+    nflush(N, rec0);
+#pragma unroll
+    for (int s = 0; s < NS; ++s) {
+      A.cnt[s] = N.cnt[s];
+      A.sdisc[s] = N.disc[s];
+      A.sq[s] = N.sq[s];
+      A.sp[s] = N.sp[s];
+      A.sdp[s] = N.dp[s];
+      A.sch[s] = N.ch[s];
+    }
+    A.status = status;
+  }
+  reduce_and_fold<QN_NW>(A, P, S.s_w, &S.status, &S.last);
+}
+
+// ------------------------------------------------------------- encoder
+struct EncParams {
+  ra_lineitem in;
+  ra_lineitem_narrow_out out;
+  int64_t n;
+  uint32_t* status;
+};
+
+__global__ void __launch_bounds__(256) q1_encode_kernel(const EncParams E) {
+  uint32_t st = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < E.n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t sd = E.in.shipdate[i];
+    const uint32_t rf = E.in.returnflag[i], ls = E.in.linestatus[i];
+    const uint64_t q = (uint64_t)E.in.quantity[i], p = (uint64_t)E.in.extendedprice[i];
+    const uint64_t d = (uint64_t)E.in.discount[i], t = (uint64_t)E.in.tax[i];
+    const int ri = rf == 'A' ? 0 : rf == 'N' ? 1 : rf == 'R' ? 2 : -1;
+    const int li = ls == 'F' ? 0 : ls == 'O' ? 1 : -1;
+    const bool okf = (ri >= 0) & (li >= 0);
+    const bool okn = (q < 65536u) & (p < (1u << 24)) & (d <= 100u) & (t <= 100u);
+    const bool oks = (sd >= 0) & (sd <= 65535);
+    st |= (okf ? 0u : 1u) | (okn ? 0u : 2u) | (oks ? 0u : 4u);
+    E.out.shipdate[i] = (uint16_t)(sd < 0 ? 0 : sd > 65535 ? 65535 : sd);
+    E.out.group[i] = !okf ? (uint8_t)0xFF : !okn ? (uint8_t)0xFE : (uint8_t)(2 * ri + li);
+    E.out.quantity[i] = (uint16_t)q;
+    E.out.discount[i] = (uint8_t)d;
+    E.out.tax[i] = (uint8_t)t;
+    E.out.extendedprice[i] = (uint32_t)p;
+  }
+  st = __reduce_or_sync(0xffffffffu, st);
+  if ((threadIdx.x & 31) == 0 && st) atomicOr(E.status, st);
+}
+
+bool g_qn_attr[64];
+
+}  // namespace
+
+int launch_q1_narrow(const ra_lineitem_narrow& c, int64_t n, int32_t cutoff, ra_q1_partial* d_partial,
+                     void* d_ws, cudaStream_t s, int accumulate) {
+  QnParams P;
+  P.sd = c.shipdate;
+  P.g = c.group;
+  P.q = c.quantity;
+  P.d = c.discount;
+  P.t = c.tax;
+  P.p = c.extendedprice;
+  P.n = n;
+  P.ntiles = n / QN_TILE;
+  P.cutoff = cutoff;
+  P.out = d_partial;
+  P.accumulate = accumulate;
+  P.counter = (uint32_t*)d_ws;
+  P.blocks = (Q1Block*)((char*)d_ws + 256);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (!g_qn_attr[dev]) {
+    cudaError_t e = cudaFuncSetAttribute(q1n_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)QN_SMEM);
+    if (e != cudaSuccess) return cuda_fail(e, "q1n_kernel smem attribute");
+    g_qn_attr[dev] = true;
+  }
+  int64_t grid = num_sms();
+  const int64_t need = P.ntiles > 0 ? P.ntiles : 1;
+  if (grid > need) grid = need;
+  // per-thread sums stay exact while rows/thread <= 2^17
+  const int64_t min_grid = (n >> 17) / QN_NT + 1;
+  if (grid < min_grid) grid = min_grid;
+  if (grid > Q1_MAX_GRID) return fail(RA_E_INVAL, "n too large for the Q1 grid");
+  q1n_kernel<<<(unsigned)grid, QN_NT + 32, QN_SMEM, s>>>(P);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "q1n_kernel launch");
+  return RA_OK;
+}
+
+int launch_q1_encode(const ra_lineitem& in, int64_t n, const ra_lineitem_narrow_out& out, uint32_t* d_status,
+                     cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(d_status, 0, sizeof(uint32_t), s);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(encode status)");
+  if (n == 0) return RA_OK;
+  EncParams E;
+  E.in = in;
+  E.out = out;
+  E.n = n;
+  E.status = d_status;
+  int64_t grid = (n + 255) / 256;
+  const int64_t cap = (int64_t)num_sms() * 8;
+  if (grid > cap) grid = cap;
+  q1_encode_kernel<<<(unsigned)grid, 256, 0, s>>>(E);
+  count_launch();
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "q1_encode_kernel launch");
+  return RA_OK;
+}
+
+}  // namespace ra

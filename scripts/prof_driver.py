@@ -46,8 +46,28 @@ def main():
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / reps
             print(f"q1 SF{sf}: {ms:.4f} ms  {38 * n / ms / 1e6:.1f} GB/s  {n / ms * 1e3:.3e} rows/s")
+            enc, _ = R.q1_encode(cols)
             del cols
             torch.cuda.empty_cache()
+            for _ in range(3):
+                R.q1_narrow(enc)
+            e0.record()
+            for _ in range(reps):
+                R.q1_narrow(enc)
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / reps
+            print(f"q1 narrow SF{sf}: {ms:.4f} ms  {11 * n / ms / 1e6:.1f} GB/s  {n / ms * 1e3:.3e} rows/s")
+            cols = enc
+            torch.cuda.empty_cache()
+    elif what == "q1n":  # narrow Q1 at SF10 (for ncu)
+        n = ragen.rows_for_sf(10)
+        cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+                for name, dt in ragen.LINEITEM_COLUMNS}
+        ragen.lineitem_dev(5, ragen.parts_for_sf(10), cols)
+        enc, _ = R.q1_encode(cols)
+        for _ in range(reps):
+            R.q1_narrow(enc)
     elif what == "q1":
         n = ragen.rows_for_sf(10)
         cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")

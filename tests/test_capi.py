@@ -28,6 +28,7 @@ def test_struct_sizes_match_header_layout():
     assert ctypes.sizeof(R.ra_q1_group) == 64
     assert ctypes.sizeof(R.ra_q1_partial) == 16 + 6 * 64
     assert ctypes.sizeof(R.ra_q1_row) == 8 + 8 * 8 + 3 * 8
+    assert ctypes.sizeof(R.ra_lineitem_narrow) == ctypes.sizeof(R.ra_lineitem_narrow_out) == 6 * 8
     assert R.ra_version() == 1
 
 
@@ -67,6 +68,21 @@ def test_argument_errors_without_gpu():
         R.ra_q1(li, 1 << 32, 10471, 4096, 256, 1 << 20, 0)
     assert e.value.code == R.RA_E_INVAL
     assert "n=" in R.ra_last_error()
+    nl = R.ra_lineitem_narrow()
+    with pytest.raises(R.RAError) as e:  # null narrow columns
+        R.ra_q1_narrow(nl, 5, 10471, 4096, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    nl = R.ra_lineitem_narrow(*([4096 + 8] * 6))
+    with pytest.raises(R.RAError) as e:  # narrow columns not 16-B aligned
+        R.ra_q1_narrow(nl, 5, 10471, 4096, 256, 1 << 20, 0)
+    assert e.value.code == R.RA_E_INVAL
+    nl = R.ra_lineitem_narrow(*([4096] * 6))
+    with pytest.raises(R.RAError) as e:  # workspace too small
+        R.ra_q1_narrow(nl, 5, 10471, 4096, 256, 16, 0)
+    assert e.value.code == R.RA_E_WORKSPACE
+    with pytest.raises(R.RAError) as e:  # encode: null output columns
+        R.ra_q1_encode(R.ra_lineitem(*([4096] * 7)), 5, R.ra_lineitem_narrow_out(), 4096, 0)
+    assert e.value.code == R.RA_E_INVAL
 
 
 SLOT = {(ord(rf), ord(ls)): 2 * i + j for i, rf in enumerate("ANR") for j, ls in enumerate("FO")}

@@ -1,0 +1,171 @@
+"""GPU parity of the narrow Q1 encoding through the C-ABI.
+
+* ra_q1_encode: the narrow columns equal a numpy re-encoding of the wide ones
+  (bit-exact), and out-of-domain rows are reported in the status word.
+* ra_q1_narrow(encode(cols)): the partial, finalised, equals the CPU oracle's
+  Q1 over the WIDE columns bit for bit (sums, 128-bit disc_price/charge, AVG
+  doubles) — the encoding is lossless on its domain.
+* out-of-domain narrow rows (group > 5, discount/tax > 100, price >= 2^24)
+  set status bits and are not accumulated (oracle over the remaining rows).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import ragen
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+CUTOFF = 10471
+KEYS = ("count_order", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "sum_disc",
+        "avg_qty", "avg_price", "avg_disc")
+RI = {ord("A"): 0, ord("N"): 1, ord("R"): 2}
+LI = {ord("F"): 0, ord("O"): 1}
+
+
+@pytest.fixture(scope="module")
+def R():
+    import paper_conf_ipps_wudwcyc12_b200 as R
+    return R
+
+
+def dev(cols):
+    return {k: torch.from_numpy(np.ascontiguousarray(v)).cuda() for k, v in cols.items()}
+
+
+def np_encode(cols):
+    """Test-side expected narrow columns (the ra.h layout, written out)."""
+    g = np.array([2 * RI[a] + LI[b] for a, b in zip(cols["returnflag"].tolist(), cols["linestatus"].tolist())],
+                 dtype=np.uint8)
+    return {"shipdate": cols["shipdate"].astype(np.uint16), "group": g,
+            "quantity": cols["quantity"].astype(np.uint16), "discount": cols["discount"].astype(np.uint8),
+            "tax": cols["tax"].astype(np.uint8), "extendedprice": cols["extendedprice"].astype(np.uint32)}
+
+
+def run_narrow(R, ncols, cutoff=CUTOFF):
+    part = R.q1_narrow(ncols, cutoff)
+    torch.cuda.synchronize()
+    raw = bytes(part.cpu().numpy().tobytes())
+    rows, rc = R.q1_finalize(raw)
+    return rows, rc, R.partials_from_bytes(raw)[0]
+
+
+def assert_same(rows, exp):
+    assert [(r["returnflag"], r["linestatus"]) for r in rows] == [(e["returnflag"], e["linestatus"]) for e in exp]
+    for r, e in zip(rows, exp):
+        for k in KEYS:
+            assert r[k] == e[k], (r["returnflag"], r["linestatus"], k, r[k], e[k])
+
+
+@pytest.mark.parametrize("n", [0, 1, 5, 1023, 1024, 1025, 4097, 100003, 1_000_000])
+def test_encode_matches_numpy_and_q1_matches_oracle(R, n):
+    cols = ragen.lineitem(51 + n, n, 20000)
+    enc, st = R.q1_encode(dev(cols))
+    torch.cuda.synchronize()
+    assert int(st.item()) == 0
+    exp_enc = np_encode(cols)
+    for k, v in exp_enc.items():
+        assert np.array_equal(enc[k].cpu().numpy(), v), k
+    exp, _ = oracle.q1(cols, CUTOFF)
+    rows, rc, part = run_narrow(R, enc)
+    assert rc == R.RA_OK and part.status == 0 and part.rows == n
+    assert_same(rows, exp)
+
+
+@pytest.mark.parametrize("cutoff", [-1, 0, 8035, 8036, 9298, 10471, 10561, 65535, 65536, 2**31 - 1, -(2**31)])
+def test_cutoffs(R, cutoff):
+    cols = ragen.lineitem(52, 300007, 20000)
+    enc, _ = R.q1_encode(dev(cols))
+    exp, _ = oracle.q1(cols, cutoff)
+    rows, rc, _ = run_narrow(R, enc, cutoff)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)
+
+
+def test_sf10_device_generated(R):
+    """BASELINE configs[2] (SF10) generated on the device, encoded, queried."""
+    n = ragen.rows_for_sf(10)
+    dcols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+             for name, dt in ragen.LINEITEM_COLUMNS}
+    ragen.lineitem_dev(3, ragen.parts_for_sf(10), dcols)
+    enc, st = R.q1_encode(dcols)
+    del dcols
+    rows, rc, _ = run_narrow(R, enc)
+    assert int(st.item()) == 0 and rc == R.RA_OK
+    exp, _ = oracle.q1(ragen.lineitem(3, n, ragen.parts_for_sf(10)), CUTOFF)
+    assert_same(rows, exp)
+
+
+def test_extreme_values_many_flushes(R):
+    """All rows in one group at the narrow maxima: the 32-bit record fields
+    reach their bounds between flushes (10 M rows > 256 per thread)."""
+    n = 10_000_000
+    cols = ragen.lineitem(53, n, 2000)
+    cols["returnflag"][:] = ord("R")
+    cols["linestatus"][:] = ord("O")
+    cols["quantity"][:] = 65535
+    cols["extendedprice"][:] = (1 << 24) - 1
+    cols["discount"][:] = 0
+    cols["discount"][::3] = 100
+    cols["tax"][:] = 100
+    enc, st = R.q1_encode(dev(cols))
+    assert int(st.item()) == 0
+    exp, _ = oracle.q1(cols, 2**31 - 1)
+    rows, rc, _ = run_narrow(R, enc, 2**31 - 1)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)
+
+
+def test_encode_reports_domain(R):
+    cols = ragen.lineitem(54, 5000, 2000)
+    for col, idx, val, bit in (("returnflag", 10, ord("Z"), 1), ("quantity", 20, 1 << 16, 2),
+                               ("extendedprice", 30, 1 << 24, 2), ("tax", 40, 101, 2), ("shipdate", 50, 70000, 4),
+                               ("shipdate", 60, -1, 4)):
+        bad = {k: v.copy() for k, v in cols.items()}
+        bad[col][idx] = val
+        enc, st = R.q1_encode(dev(bad))
+        torch.cuda.synchronize()
+        assert int(st.item()) == bit, (col, int(st.item()))
+        g = enc["group"].cpu().numpy()
+        if bit == 1:
+            assert g[idx] == 0xFF
+        elif bit == 2:
+            assert g[idx] == 0xFE
+
+
+def test_narrow_domain_rows_not_accumulated(R):
+    n = 200_001
+    cols = ragen.lineitem(55, n, 20000)
+    enc = np_encode(cols)
+    bad_g, bad_d, bad_p = 7, 11, 13
+    enc["group"][bad_g] = 6
+    enc["discount"][bad_d] = 101
+    enc["extendedprice"][bad_p] = 1 << 24
+    rows, rc, part = run_narrow(R, dev(enc), 10561)
+    assert part.status == 3 and rc == R.RA_E_DOMAIN
+    keep = np.ones(n, bool)
+    keep[[bad_g, bad_d, bad_p]] = False
+    exp, _ = oracle.q1({k: v[keep] for k, v in cols.items()}, 10561)
+    assert_same(rows, exp)
+
+
+def test_repeated_launches_and_shards(R):
+    n = 700_001
+    cols = ragen.lineitem(56, n, 20000)
+    exp, _ = oracle.q1(cols, CUTOFF)
+    enc, _ = R.q1_encode(dev(cols))
+    parts = [R.q1_narrow(enc, CUTOFF) for _ in range(10)]
+    torch.cuda.synchronize()
+    for p in parts:
+        rows, rc = R.q1_finalize(bytes(p.cpu().numpy().tobytes()))
+        assert_same(rows, exp)
+    # row-range shards at 16-row-aligned cuts -> exact merge
+    raws = b""
+    for a, b in ((0, 16 * 1000), (16 * 1000, 16 * 30001), (16 * 30001, n)):
+        p = R.q1_narrow({k: v[a:b] for k, v in enc.items()}, CUTOFF)
+        torch.cuda.synchronize()
+        raws += p.cpu().numpy().tobytes()
+    rows, rc = R.q1_finalize(raws)
+    assert rc == R.RA_OK
+    assert_same(rows, exp)

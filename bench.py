@@ -143,6 +143,21 @@ def peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def read_peak():
+    """Read-only HBM stream peak measured by scripts/micro/stream_bw.cu (committed
+    under profiles/): context for read-dominated kernels, whose fraction of the
+    copy (read+write) peak in MEASURED_PEAKS.json can exceed 1."""
+    p = os.path.join(ROOT, "profiles", "r01_stream_bw.txt")
+    if not os.path.exists(p):
+        return None
+    best = 0.0
+    with open(p) as f:
+        for line in f:
+            if line.startswith("bulk") and "GB/s" in line:
+                best = max(best, float(line.split(":")[1].split()[0]))
+    return best or None
+
+
 def ncu_traffic(key: str):
     """dram bytes per launch from the committed ncu --set full capture, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -358,12 +373,40 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
         raw = parts[0].cpu().numpy().tobytes()
         rows, rc = R.q1_finalize(raw)
         ach = 38 * m / (qkms * 1e-3) / 1e9
+        res = {"rows": N, "rows_per_s": (N if shard else m) / (qms * 1e-3), "ms_per_step": qms,
+               "kernel_ms": qkms, "groups": len(rows), "finalize_rc": rc,
+               "roofline": {"kernel": "q1_tma_kernel", "bound": "hbm", "achieved": ach, "peak": peak,
+                            "unit": "GB/s", "frac": ach / peak, "algorithmic_bytes_per_launch": 38 * m,
+                            "traffic": ncu_traffic(f"q1_sf{int(sf)}"), "read_stream_peak": read_peak(),
+                            "frac_of_read_stream_peak": ach / read_peak() if read_peak() else None}}
+
+        # f4: the same rows re-encoded narrow (11 B/row), same partial / finalize
+        enc, est = R.q1_encode(cols, stream=torch.cuda.current_stream())
         del cols
-        return {"rows": N, "rows_per_s": (N if shard else m) / (qms * 1e-3), "ms_per_step": qms,
-                "kernel_ms": qkms, "groups": len(rows), "finalize_rc": rc,
-                "roofline": {"kernel": "q1_fused_kernel", "bound": "hbm", "achieved": ach, "peak": peak,
-                             "unit": "GB/s", "frac": ach / peak, "algorithmic_bytes_per_launch": 38 * m,
-                             "traffic": ncu_traffic(f"q1_sf{int(sf)}")}}
+        assert int(est.item()) == 0
+        hn = R.ra_lineitem_narrow(*[enc[name].data_ptr() for name, _ in R.NARROW_COLUMNS])
+
+        def nkern(i):
+            R.ra_q1_narrow(hn, m, R.Q1_CUTOFF_DELTA90, part.data_ptr(), wsq.data_ptr(), wsq_b, sh)
+
+        def nstep(i, kernel_done=False):
+            if not kernel_done:
+                nkern(i)
+            if D.pg and shard:
+                parts[0] = rdist.gather_partials(part)
+
+        nms, nkms = timed(torch, D, nstep, 50, 5, kernel_fn=nkern)
+        nrows, nrc = R.q1_finalize(parts[0].cpu().numpy().tobytes())
+        assert nrows == rows, "narrow and wide Q1 disagree"
+        nach = 11 * m / (nkms * 1e-3) / 1e9
+        res["narrow"] = {"rows_per_s": (N if shard else m) / (nms * 1e-3), "ms_per_step": nms, "kernel_ms": nkms,
+                         "bytes_per_row": 11, "same_result_as_wide": True,
+                         "roofline": {"kernel": "q1n_kernel", "bound": "hbm", "achieved": nach, "peak": peak,
+                                      "unit": "GB/s", "frac": nach / peak, "algorithmic_bytes_per_launch": 11 * m,
+                                      "traffic": ncu_traffic(f"q1n_sf{int(sf)}"),
+                                      "note": "issue/shared-memory bound (per-row group-record update), see DESIGN.md"}}
+        del enc
+        return res
 
     if D.world == 1:
         ex["q1_sf10"] = q1_bench(10, False)
@@ -389,11 +432,29 @@ def q1_e2e(args, D, torch, R, sf):
     part = R.q1_fission_run(h, chunk, streams)
     ms, _ = timed(torch, D, lambda i, kernel_done=False: R.q1_fission_run(h, chunk, streams), 3, 1)
     rows, rc = R.q1_finalize(bytes(part))
+    res = {"value": N / (ms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 38 * N,
+           "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": ms,
+           "pcie_h2d_gbs": 38 * N / (ms * 1e-3) / 1e9, "groups": len(rows), "finalize_rc": rc,
+           "path": "ra_q1_fission_run: pinned host columns, chunk 2^22 rows, 3 streams"}
+    # f1 x f4: the same table held narrow (11 B/row) in pinned host memory
+    dcols = {k: v.cuda() for k, v in h.items()}
     del h
-    return {"value": N / (ms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 38 * N,
-            "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": ms,
-            "pcie_h2d_gbs": 38 * N / (ms * 1e-3) / 1e9, "groups": len(rows), "finalize_rc": rc,
-            "path": "ra_q1_fission_run: pinned host columns, chunk 2^22 rows, 3 streams"}
+    enc, st = R.q1_encode(dcols)
+    del dcols
+    assert int(st.item()) == 0
+    hn = {k: v.cpu().pin_memory() for k, v in enc.items()}
+    del enc
+    chunk_n = 1 << 23
+    npart = R.q1_narrow_fission_run(hn, chunk_n, streams)
+    nms, _ = timed(torch, D, lambda i, kernel_done=False: R.q1_narrow_fission_run(hn, chunk_n, streams), 3, 1)
+    nrows, nrc = R.q1_finalize(bytes(npart))
+    assert nrows == rows, "narrow fission and wide fission disagree"
+    res["narrow"] = {"value": N / (nms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 11 * N,
+                     "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": nms,
+                     "pcie_h2d_gbs": 11 * N / (nms * 1e-3) / 1e9,
+                     "path": "ra_q1_narrow_fission_run: pinned host narrow columns, chunk 2^23 rows, 3 streams"}
+    del hn
+    return res
 
 
 def cpu_baseline(x, preds, n):

@@ -301,6 +301,17 @@ int ra_q1_encode(const ra_lineitem* h_cols, int64_t n, const ra_lineitem_narrow_
 int ra_q1_narrow(const ra_lineitem_narrow* h_cols, int64_t n, int32_t shipdate_cutoff,
                  ra_q1_partial* d_partial, void* d_ws, size_t ws_bytes, ra_stream_t stream);
 
+/* Host-resident narrow Q1 under kernel fission (f1 x f4): as
+ * ra_q1_fission_run, but h_cols holds PINNED host narrow columns (11 B/row
+ * over PCIe instead of 38).  Result identical to ra_q1_narrow on the whole
+ * table.  Synchronous.  d_ws: ra_q1_narrow_fission_workspace_bytes, 256-B
+ * aligned. */
+size_t ra_q1_narrow_fission_workspace_bytes(int64_t chunk_rows, int n_streams);
+
+int ra_q1_narrow_fission_run(const ra_lineitem_narrow* h_cols, int64_t n, int32_t shipdate_cutoff,
+                             int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
+                             ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes);
+
 #ifdef __cplusplus
 }
 #endif

@@ -21,7 +21,7 @@ from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, r
                   ra_fission_workspace_bytes, ra_lineitem, ra_q1, ra_q1_finalize, ra_q1_partial,
                   ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
                   ra_select_chain, ra_select_workspace_bytes, ra_lineitem_narrow, ra_lineitem_narrow_out,
-                  ra_q1_encode, ra_q1_narrow)
+                  ra_q1_encode, ra_q1_narrow, ra_q1_narrow_fission_run, ra_q1_narrow_fission_workspace_bytes)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
@@ -207,4 +207,27 @@ def q1_fission_run(h_cols, chunk_rows: int, streams, cutoff: int = Q1_CUTOFF_DEL
     part = ra_q1_partial()
     ra_q1_fission_run(lineitem_struct(h_cols), n, int(cutoff), chunk_rows, sarr, S, part, ws.data_ptr(),
                       ws.numel())
+    return part
+
+
+def q1_narrow_fission_run(h_cols, chunk_rows: int, streams, cutoff: int = Q1_CUTOFF_DELTA90, device=None):
+    """Host-resident narrow Q1 under kernel fission (synchronous, f1 x f4).
+
+    ``h_cols``: dict of pinned contiguous CPU tensors (NARROW_COLUMNS).
+    Returns the whole query's ``ra_q1_partial``.
+    """
+    torch = _torch()
+    n = h_cols["shipdate"].numel()
+    for name, _ in NARROW_COLUMNS:
+        t = h_cols[name]
+        if t.numel() != n or t.device.type != "cpu" or not t.is_contiguous() or (n and not t.is_pinned()):
+            raise ValueError(f"h_cols[{name!r}] must be a pinned contiguous CPU tensor of {n} rows")
+    chunk_rows = max(1, min(int(chunk_rows), max(1, n)))
+    device = device or torch.device("cuda", torch.cuda.current_device())
+    S = len(streams)
+    sarr = (ctypes.c_void_p * S)(*[_stream_handle(s) for s in streams])
+    ws = workspace(device, f"q1n_fission_{S}", ra_q1_narrow_fission_workspace_bytes(chunk_rows, S))
+    part = ra_q1_partial()
+    h = ra_lineitem_narrow(*[h_cols[name].data_ptr() for name, _ in NARROW_COLUMNS])
+    ra_q1_narrow_fission_run(h, n, int(cutoff), chunk_rows, sarr, S, part, ws.data_ptr(), ws.numel())
     return part

@@ -122,6 +122,8 @@ _SIGS = {
     "ra_q1_fission_run": ([_vp, _i64, ctypes.c_int32, _i64, _vp, _i32, _vp, _vp, _sz], _i32),
     "ra_q1_encode": ([_vp, _i64, _vp, _vp, _vp], _i32),
     "ra_q1_narrow": ([_vp, _i64, ctypes.c_int32, _vp, _vp, _sz, _vp], _i32),
+    "ra_q1_narrow_fission_workspace_bytes": ([_i64, _i32], _sz),
+    "ra_q1_narrow_fission_run": ([_vp, _i64, ctypes.c_int32, _i64, _vp, _i32, _vp, _vp, _sz], _i32),
 }
 for _name, (_args, _res) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -222,6 +224,16 @@ def ra_q1_encode(h_cols: ra_lineitem, n: int, h_out: ra_lineitem_narrow_out, d_s
 def ra_q1_narrow(h_cols: ra_lineitem_narrow, n: int, cutoff: int, d_partial: int, d_ws: int, ws_bytes: int,
                  stream: int) -> None:
     _check(_lib.ra_q1_narrow(ctypes.byref(h_cols), n, cutoff, d_partial, d_ws, ws_bytes, stream))
+
+
+def ra_q1_narrow_fission_workspace_bytes(chunk_rows: int, n_streams: int) -> int:
+    return int(_lib.ra_q1_narrow_fission_workspace_bytes(chunk_rows, n_streams))
+
+
+def ra_q1_narrow_fission_run(h_cols: ra_lineitem_narrow, n: int, cutoff: int, chunk_rows: int, streams,
+                             n_streams: int, h_partial, d_ws: int, ws_bytes: int) -> None:
+    _check(_lib.ra_q1_narrow_fission_run(ctypes.byref(h_cols), n, cutoff, chunk_rows, streams, n_streams,
+                                         ctypes.byref(h_partial), d_ws, ws_bytes))
 
 
 def make_preds(preds):

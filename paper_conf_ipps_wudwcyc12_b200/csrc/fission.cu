@@ -173,24 +173,28 @@ RA_API int ra_fission_run(const int32_t* h_in, int64_t n, const ra_pred* h_preds
 namespace ra {
 namespace {
 
-// Per-stream region: the chunk's seven columns, the Q1 kernel workspace and
-// the stream's running partial.
+// Per-stream region: the chunk's columns (each 256-B aligned), the Q1 kernel
+// workspace and the stream's running partial.
 struct Q1Region {
-  size_t sd, rf, ls, dec, ws, part, total;
+  size_t col[8];
+  size_t ws, part, total;
 };
 
-Q1Region q1_region(int64_t chunk_rows) {
+Q1Region q1_region(int64_t chunk_rows, const size_t* esz, int ncol) {
   Q1Region r;
-  const size_t c = (size_t)chunk_rows;
-  r.sd = 0;
-  r.rf = r.sd + round256(c * 4);
-  r.ls = r.rf + round256(c);
-  r.dec = r.ls + round256(c);  // 4 decimal columns, round256(c * 8) each
-  r.ws = r.dec + 4 * round256(c * 8);
+  size_t off = 0;
+  for (int j = 0; j < ncol; ++j) {
+    r.col[j] = off;
+    off += round256((size_t)chunk_rows * esz[j]);
+  }
+  r.ws = off;
   r.part = r.ws + round256(q1_ws_bytes());
   r.total = r.part + round256(sizeof(ra_q1_partial));
   return r;
 }
+
+constexpr size_t WIDE_ESZ[7] = {4, 1, 1, 8, 8, 8, 8};    // ra_lineitem order
+constexpr size_t NARROW_ESZ[6] = {2, 1, 2, 1, 1, 4};     // ra_lineitem_narrow order
 
 // exact slotwise sum (the shard merge of ra_q1_finalize, without finalising)
 void q1_merge(ra_q1_partial& acc, const ra_q1_partial& p) {
@@ -217,38 +221,37 @@ void q1_merge(ra_q1_partial& acc, const ra_q1_partial& p) {
 }  // namespace
 }  // namespace ra
 
-RA_API size_t ra_q1_fission_workspace_bytes(int64_t chunk_rows, int n_streams) {
-  if (chunk_rows <= 0 || n_streams <= 0) return 0;
-  return (size_t)n_streams * q1_region(chunk_rows).total;
-}
+namespace ra {
+namespace {
 
-RA_API int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff,
-                             int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
-                             ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes) {
-  clear_error();
-  if (!h_cols || !h_partial || !streams) return fail(RA_E_INVAL, "null argument");
+// Q1 under fission for any column layout: chunk c -> stream c % S: H2D of its
+// column slices -> Q1 kernel accumulating into the stream's partial; the S
+// partials are merged exactly at the end.  `launch(cols, len, partial, ws, st)`
+// enqueues the layout's kernel in accumulate mode.
+template <typename Launch>
+int q1_fission_generic(const void* const* cols, const char* const* names, const size_t* esz, int ncol, int64_t n,
+                       int64_t chunk_rows, const ra_stream_t* streams, int n_streams, ra_q1_partial* h_partial,
+                       void* d_ws, size_t ws_bytes, Launch launch) {
+  if (!h_partial || !streams) return fail(RA_E_INVAL, "null argument");
   if (n < 0 || n >= (int64_t)1 << 32 || chunk_rows <= 0 || n_streams <= 0)
     return fail(RA_E_INVAL, "bad sizes (n=%lld chunk_rows=%lld n_streams=%d)", (long long)n,
                 (long long)chunk_rows, n_streams);
-  const ra_lineitem& h = *h_cols;
   memset(h_partial, 0, sizeof(*h_partial));
   h_partial->n_groups = RA_Q1_GROUPS;
   if (n == 0) return RA_OK;
-  if (!h.shipdate || !h.returnflag || !h.linestatus || !h.quantity || !h.extendedprice || !h.discount || !h.tax)
-    return fail(RA_E_INVAL, "null column with n > 0");
+  for (int j = 0; j < ncol; ++j)
+    if (!cols[j]) return fail(RA_E_INVAL, "null column with n > 0");
   if (!d_ws) return fail(RA_E_INVAL, "null workspace");
   if ((uintptr_t)d_ws & 255u) return fail(RA_E_INVAL, "workspace must be 256-byte aligned");
   if (chunk_rows > n) chunk_rows = n;
-  const size_t need = ra_q1_fission_workspace_bytes(chunk_rows, n_streams);
+  const Q1Region R = q1_region(chunk_rows, esz, ncol);
+  const size_t need = (size_t)n_streams * R.total;
   if (ws_bytes < need) return fail(RA_E_WORKSPACE, "q1 fission workspace %zu < required %zu", ws_bytes, need);
-  const void* cols[7] = {h.shipdate, h.returnflag, h.linestatus, h.quantity, h.extendedprice, h.discount, h.tax};
-  const char* names[7] = {"shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax"};
-  for (int j = 0; j < 7; ++j) {
+  for (int j = 0; j < ncol; ++j) {
     int rc = check_pinned(cols[j], names[j], nullptr);
     if (rc) return rc;
   }
   const int S = n_streams;
-  const Q1Region R = q1_region(chunk_rows);
   int result = RA_OK;
   // zero each stream's running partial and its Q1 ticket word (the region
   // layout moves with chunk_rows)
@@ -266,24 +269,15 @@ RA_API int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipd
     const int64_t len = (n - r0 < chunk_rows) ? (n - r0) : chunk_rows;
     char* base = (char*)d_ws + (size_t)s * R.total;
     cudaStream_t st = (cudaStream_t)streams[s];
-    ra_lineitem d;
-    d.shipdate = (const int32_t*)(base + R.sd);
-    d.returnflag = (const uint8_t*)(base + R.rf);
-    d.linestatus = (const uint8_t*)(base + R.ls);
-    d.quantity = (const int64_t*)(base + R.dec);
-    d.extendedprice = (const int64_t*)(base + R.dec + round256((size_t)chunk_rows * 8));
-    d.discount = (const int64_t*)(base + R.dec + 2 * round256((size_t)chunk_rows * 8));
-    d.tax = (const int64_t*)(base + R.dec + 3 * round256((size_t)chunk_rows * 8));
-    const void* dst[7] = {d.shipdate, d.returnflag, d.linestatus, d.quantity, d.extendedprice, d.discount, d.tax};
-    const size_t esz[7] = {4, 1, 1, 8, 8, 8, 8};
-    for (int j = 0; j < 7 && result == RA_OK; ++j) {
-      cudaError_t e = cudaMemcpyAsync((void*)dst[j], (const char*)cols[j] + r0 * esz[j], (size_t)len * esz[j],
+    for (int j = 0; j < ncol && result == RA_OK; ++j) {
+      cudaError_t e = cudaMemcpyAsync(base + R.col[j], (const char*)cols[j] + r0 * esz[j], (size_t)len * esz[j],
                                       cudaMemcpyHostToDevice, st);
       if (e != cudaSuccess) result = cuda_fail(e, "H2D q1 chunk column");
     }
     if (result != RA_OK) break;
-    result = launch_q1(d, len, shipdate_cutoff, (ra_q1_partial*)(base + R.part), base + R.ws,
-                       R.part - R.ws, st, /*accumulate=*/1);
+    void* dcols[8];
+    for (int j = 0; j < ncol; ++j) dcols[j] = base + R.col[j];
+    result = launch(dcols, len, (ra_q1_partial*)(base + R.part), base + R.ws, st);
   }
   std::vector<ra_q1_partial> parts(S);
   for (int s = 0; s < S; ++s) {
@@ -300,4 +294,62 @@ RA_API int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipd
   for (int s = 0; s < S && s < C; ++s) q1_merge(*h_partial, parts[s]);
   h_partial->n_groups = RA_Q1_GROUPS;
   return RA_OK;
+}
+
+}  // namespace
+}  // namespace ra
+
+RA_API size_t ra_q1_fission_workspace_bytes(int64_t chunk_rows, int n_streams) {
+  if (chunk_rows <= 0 || n_streams <= 0) return 0;
+  return (size_t)n_streams * q1_region(chunk_rows, WIDE_ESZ, 7).total;
+}
+
+RA_API int ra_q1_fission_run(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff,
+                             int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
+                             ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes) {
+  clear_error();
+  if (!h_cols) return fail(RA_E_INVAL, "null argument");
+  const ra_lineitem& h = *h_cols;
+  const void* cols[7] = {h.shipdate, h.returnflag, h.linestatus, h.quantity, h.extendedprice, h.discount, h.tax};
+  static const char* const names[7] = {"shipdate", "returnflag", "linestatus", "quantity",
+                                       "extendedprice", "discount", "tax"};
+  return q1_fission_generic(cols, names, WIDE_ESZ, 7, n, chunk_rows, streams, n_streams, h_partial, d_ws, ws_bytes,
+                            [&](void* const* d, int64_t len, ra_q1_partial* part, void* ws, cudaStream_t st) {
+                              ra_lineitem c;
+                              c.shipdate = (const int32_t*)d[0];
+                              c.returnflag = (const uint8_t*)d[1];
+                              c.linestatus = (const uint8_t*)d[2];
+                              c.quantity = (const int64_t*)d[3];
+                              c.extendedprice = (const int64_t*)d[4];
+                              c.discount = (const int64_t*)d[5];
+                              c.tax = (const int64_t*)d[6];
+                              return launch_q1(c, len, shipdate_cutoff, part, ws, q1_ws_bytes(), st, 1);
+                            });
+}
+
+RA_API size_t ra_q1_narrow_fission_workspace_bytes(int64_t chunk_rows, int n_streams) {
+  if (chunk_rows <= 0 || n_streams <= 0) return 0;
+  return (size_t)n_streams * q1_region(chunk_rows, NARROW_ESZ, 6).total;
+}
+
+RA_API int ra_q1_narrow_fission_run(const ra_lineitem_narrow* h_cols, int64_t n, int32_t shipdate_cutoff,
+                                    int64_t chunk_rows, const ra_stream_t* streams, int n_streams,
+                                    ra_q1_partial* h_partial, void* d_ws, size_t ws_bytes) {
+  clear_error();
+  if (!h_cols) return fail(RA_E_INVAL, "null argument");
+  const ra_lineitem_narrow& h = *h_cols;
+  const void* cols[6] = {h.shipdate, h.group, h.quantity, h.discount, h.tax, h.extendedprice};
+  static const char* const names[6] = {"shipdate", "group", "quantity", "discount", "tax", "extendedprice"};
+  return q1_fission_generic(cols, names, NARROW_ESZ, 6, n, chunk_rows, streams, n_streams, h_partial, d_ws,
+                            ws_bytes,
+                            [&](void* const* d, int64_t len, ra_q1_partial* part, void* ws, cudaStream_t st) {
+                              ra_lineitem_narrow c;
+                              c.shipdate = (const uint16_t*)d[0];
+                              c.group = (const uint8_t*)d[1];
+                              c.quantity = (const uint16_t*)d[2];
+                              c.discount = (const uint8_t*)d[3];
+                              c.tax = (const uint8_t*)d[4];
+                              c.extendedprice = (const uint32_t*)d[5];
+                              return launch_q1_narrow(c, len, shipdate_cutoff, part, ws, st, 1);
+                            });
 }

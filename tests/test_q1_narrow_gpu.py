@@ -169,3 +169,24 @@ def test_repeated_launches_and_shards(R):
     rows, rc = R.q1_finalize(raws)
     assert rc == R.RA_OK
     assert_same(rows, exp)
+
+
+@pytest.mark.parametrize("n,chunk,S", [(1, 1, 1), (5000, 1024, 3), (1_000_003, 1 << 16, 3), (1_000_003, 999_999, 2),
+                                       (3_000_017, 1 << 20, 4)])
+def test_narrow_fission_matches_oracle_and_device(R, n, chunk, S):
+    """f1 x f4: pinned narrow host columns streamed in chunks; the merged
+    partial equals the oracle over the wide rows and the device-resident
+    narrow partial byte for byte."""
+    import ctypes
+    cols = ragen.lineitem(57 + n, n, 200000)
+    enc = np_encode(cols)
+    h = {k: torch.from_numpy(v).pin_memory() for k, v in enc.items()}
+    part = R.q1_narrow_fission_run(h, chunk, [torch.cuda.Stream() for _ in range(S)])
+    rows, rc = R.q1_finalize(bytes(part))
+    exp, _ = oracle.q1(cols, CUTOFF)
+    assert rc == R.RA_OK and part.rows == n
+    assert_same(rows, exp)
+    dpart = R.q1_narrow(dev(enc), CUTOFF)
+    torch.cuda.synchronize()
+    assert bytes(part) == dpart.cpu().numpy().tobytes()
+    assert ctypes.sizeof(part) == dpart.numel()

@@ -61,6 +61,8 @@ def lib() -> ctypes.CDLL:
             f.restype = i64
         L.oracle_select_chunked.argtypes = [vp, i64, vp, i32, i64, vp]
         L.oracle_select_chunked.restype = i64
+        L.oracle_select_rows.argtypes = [vp, i64, vp, i32, i32, vp, vp, vp, vp]
+        L.oracle_select_rows.restype = i64
         L.oracle_q1.argtypes = [vp, vp, vp, vp, vp, vp, vp, i64, ctypes.c_int32, vp, vp]
         L.oracle_q1.restype = i32
         L.oracle_q1_row_size.restype = i32
@@ -112,6 +114,30 @@ def select_chunked(x, preds, chunk: int) -> np.ndarray:
     if m < 0:
         raise ValueError(f"oracle_select_chunked failed ({m})")
     return out[:m].copy()
+
+
+def select_rows(key, preds, payloads=()):
+    """SELECT over a multi-column relation (Table I): the predicate chain on
+    the int32 key column; returns ``(rowids int64, [payload[rowids] ...])``
+    with rows in input order.  Payload columns are 4- or 8-byte arrays."""
+    key = _as_i32(key)
+    P = _preds(preds)
+    cols = [np.ascontiguousarray(c) for c in payloads]
+    for c in cols:
+        if c.size != key.size or c.dtype.itemsize not in (4, 8):
+            raise ValueError("payload columns must match the key length and be 4- or 8-byte")
+    m = len(cols)
+    rowids = np.empty(max(1, key.size), dtype=np.int64)
+    outs = [np.empty(max(1, key.size), dtype=c.dtype) for c in cols]
+    cp = (ctypes.c_void_p * max(1, m))(*[c.ctypes.data for c in cols])
+    eb = (ctypes.c_int32 * max(1, m))(*[c.dtype.itemsize for c in cols])
+    op = (ctypes.c_void_p * max(1, m))(*[o.ctypes.data for o in outs])
+    cnt = lib().oracle_select_rows(key.ctypes.data, key.size, ctypes.addressof(P), len(preds), m,
+                                   ctypes.addressof(cp), ctypes.addressof(eb), rowids.ctypes.data,
+                                   ctypes.addressof(op))
+    if cnt < 0:
+        raise ValueError(f"oracle_select_rows failed ({cnt})")
+    return rowids[:cnt].copy(), [o[:cnt].copy() for o in outs]
 
 
 def _i128(lo: int, hi: int) -> int:

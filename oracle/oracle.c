@@ -114,6 +114,38 @@ ORACLE_API int64_t oracle_select_chunked(const int32_t* x, int64_t n, const orac
   return total;
 }
 
+/* SELECT over a multi-column relation (Table I: "select
+ * [field.0==2] x -> (2,False,b)" returns whole tuples; the first field is the
+ * key).  Column store: `key` is field 0, cols[0..m) are further fields of
+ * elem_bytes[j] bytes each (4 or 8).  A row is kept iff every predicate holds
+ * on its key; kept rows come out in input order (L481-483) as their row index
+ * (rowids, may be NULL) and as each field's value (outs[j], may be NULL).
+ * With k = 0 every row is kept, which is PROJECT (Table I:
+ * "project [0,2] x") when cols names the projected fields.  Returns the
+ * number kept, -1 for an invalid predicate or element size. */
+ORACLE_API int64_t oracle_select_rows(const int32_t* key, int64_t n, const oracle_pred* P, int k, int m,
+                                      const void* const* cols, const int32_t* elem_bytes, int64_t* rowids,
+                                      void* const* outs) {
+  for (int j = 0; j < k; ++j)
+    if (oracle_cmp(P[j].op, 0, P[j].value) < 0) return -1;
+  for (int j = 0; j < m; ++j)
+    if (elem_bytes[j] != 4 && elem_bytes[j] != 8) return -1;
+  int64_t count = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    int keep = 1;
+    for (int j = 0; j < k; ++j)
+      if (!oracle_cmp(P[j].op, key[i], P[j].value)) keep = 0;
+    if (!keep) continue;
+    if (rowids) rowids[count] = i;
+    for (int j = 0; j < m; ++j)
+      if (outs && outs[j])
+        memcpy((char*)outs[j] + count * elem_bytes[j], (const char*)cols[j] + i * elem_bytes[j],
+               (size_t)elem_bytes[j]);
+    count++;
+  }
+  return count;
+}
+
 /* ------------------------------------------------------------------ Q1
  * TPC-H Q1 (EXT:TPC-H, restated SURVEY C8; the paper's plan Fig 17(a),
  * §V: SELECT on shipdate, JOINs assembling seven columns, SORT by

@@ -47,3 +47,15 @@ def rows_to_columns(rows):
         "discount": np.array([r[5] for r in rows], dtype=np.int64),
         "tax": np.array([r[6] for r in rows], dtype=np.int64),
     }
+
+
+def table1_tuples():
+    """Table I's relation as three int32 columns, with its PROJECT and SELECT results."""
+    d = dict(_lines("table1_tuples.txt"))
+    cols = [[int(v) for v in d[f"field{j}"]] for j in range(3)]
+    sel = (d["select_pred"][0], int(d["select_pred"][1]))
+    sel_out = tuple(int(v) for v in d["select_out"])
+    proj_fields = [int(v) for v in d["project_fields"]]
+    po = [int(v) for v in d["project_out"]]
+    proj_out = [tuple(po[i:i + len(proj_fields)]) for i in range(0, len(po), len(proj_fields))]
+    return cols, sel, sel_out, proj_fields, proj_out

@@ -94,3 +94,41 @@ def test_fused_equals_unfused_and_chunks(s, k):
 def test_invalid_op_rejected():
     with pytest.raises(ValueError):
         oracle.select([1, 2], [(9, 0)])
+
+
+# ---------------------------------------------------------------- tuples (f3)
+def test_table1_tuple_select_and_project():
+    """Table I: select [field.0==2] x -> (2,False,b); project [0,2] x -> {(3,a),(4,a),(2,b)}."""
+    from golden_io import table1_tuples
+    cols, sel, sel_out, proj_fields, proj_out = table1_tuples()
+    f = [np.array(c, dtype=np.int32) for c in cols]
+    rowids, outs = oracle.select_rows(f[0], [sel], f)
+    assert rowids.tolist() == [2]
+    assert tuple(int(o[0]) for o in outs) == sel_out
+    rowids, outs = oracle.select_rows(f[0], [], [f[j] for j in proj_fields])  # k = 0: PROJECT
+    assert rowids.tolist() == [0, 1, 2]
+    assert list(zip(*[o.tolist() for o in outs])) == proj_out
+
+
+@settings(max_examples=200, deadline=None)
+@given(rows=st.lists(st.tuples(st.one_of(I32, st.integers(-4, 4)), I32, st.integers(-2**63, 2**63 - 1)),
+                     max_size=50),
+       preds=st.lists(st.tuples(st.sampled_from(OPS), st.one_of(I32, st.integers(-4, 4))), max_size=4))
+def test_select_rows_equals_brute_force(rows, preds):
+    key = np.array([r[0] for r in rows], dtype=np.int32)
+    a = np.array([r[1] for r in rows], dtype=np.int32)
+    b = np.array([r[2] for r in rows], dtype=np.int64)
+    exp = [(i, r[1], r[2]) for i, r in enumerate(rows) if all(PY_CMP[op](r[0], v) for op, v in preds)]
+    rowids, (oa, ob) = oracle.select_rows(key, preds, [a, b])
+    assert list(zip(rowids.tolist(), oa.tolist(), ob.tolist())) == exp
+
+
+def test_select_rows_matches_numpy_and_value_select():
+    x = ragen.int32_column(9, 100_003)
+    pay = np.arange(x.size, dtype=np.int64) * 7 - 3
+    preds = [("gt", -(2**30)), ("lt", 2**29), ("ne", int(x[17]))]
+    mask = (x > -(2**30)) & (x < 2**29) & (x != x[17])
+    rowids, (okey, opay) = oracle.select_rows(x, preds, [x, pay])
+    assert np.array_equal(rowids, np.flatnonzero(mask))
+    assert np.array_equal(okey, x[mask]) and np.array_equal(opay, pay[mask])
+    assert np.array_equal(okey, oracle.select(x, preds))

@@ -6,7 +6,8 @@ pipeline.  This package is the thin Python layer above it:
 
 * ``ra_*`` — one-to-one ctypes bindings of the C entry points (``_ra.py``);
 * ``select_chain``, ``q1``, ``q1_finalize``, ``fission_run``,
-  ``q1_fission_run``, ``q1_encode``, ``q1_narrow`` — conveniences
+  ``q1_fission_run``, ``q1_encode``, ``q1_narrow``, ``q1_narrow_fission_run``,
+  ``select_rows`` — conveniences
   that take torch tensors, allocate outputs/workspaces with torch (device
   memory and streams are PyTorch's; nothing else is) and call the bindings.
 
@@ -21,7 +22,8 @@ from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, r
                   ra_fission_workspace_bytes, ra_lineitem, ra_q1, ra_q1_finalize, ra_q1_partial,
                   ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
                   ra_select_chain, ra_select_workspace_bytes, ra_lineitem_narrow, ra_lineitem_narrow_out,
-                  ra_q1_encode, ra_q1_narrow, ra_q1_narrow_fission_run, ra_q1_narrow_fission_workspace_bytes)
+                  ra_q1_encode, ra_q1_narrow, ra_q1_narrow_fission_run, ra_q1_narrow_fission_workspace_bytes,
+                  ra_payload, ra_select_rows)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
@@ -75,6 +77,35 @@ def select_chain(x, preds, fused: bool = True, out=None, count=None, stream=None
     ra_select_chain(x.data_ptr(), n, P, k, int(fused), out.data_ptr(), out.numel(), count.data_ptr(),
                     ws.data_ptr(), ws.numel(), _stream_handle(stream))
     return out, count
+
+
+def select_rows(key, preds, payloads=(), rowids: bool = True, out_cap=None, stream=None):
+    """Tuple SELECT (Table I) over a CUDA int32 key column and payload columns
+    (CUDA 4- or 8-byte tensors of the same length), one fused pass.
+
+    Returns ``(rowids, outs, count)``: ``rowids[:count]`` (uint32, or None),
+    ``outs[j][:count]`` the payload fields of the selected rows in input order,
+    ``count`` a 1-element int64 CUDA tensor (not synchronised)."""
+    torch = _torch()
+    if not (key.is_cuda and key.dtype == torch.int32 and key.is_contiguous()):
+        raise ValueError("key must be a contiguous CUDA int32 tensor")
+    n, k = key.numel(), len(preds)
+    cap = n if out_cap is None else int(out_cap)
+    ids = torch.empty(max(1, cap), dtype=torch.uint32, device=key.device) if rowids else None
+    outs, pl = [], (ra_payload * max(1, len(payloads)))()
+    for j, c in enumerate(payloads):
+        if not (c.is_cuda and c.is_contiguous() and c.numel() == n and c.element_size() in (4, 8)):
+            raise ValueError("payloads must be contiguous CUDA 4/8-byte tensors of the key's length")
+        o = torch.empty(max(1, cap), dtype=c.dtype, device=key.device)
+        outs.append(o)
+        pl[j].col, pl[j].out, pl[j].elem_bytes = c.data_ptr(), o.data_ptr(), c.element_size()
+    count = torch.empty(1, dtype=torch.int64, device=key.device)
+    need = ra_select_workspace_bytes(n, k, 1)
+    ws = workspace(key.device, "select_fused", need, stream)
+    P = make_preds(preds)
+    ra_select_rows(key.data_ptr(), n, P, k, ids.data_ptr() if ids is not None else 0, pl, len(payloads), cap,
+                   count.data_ptr(), ws.data_ptr(), ws.numel(), _stream_handle(stream))
+    return ids, outs, count
 
 
 def lineitem_struct(cols) -> ra_lineitem:

@@ -30,6 +30,7 @@ RA_E_NOT_PINNED = -4
 RA_E_CUDA = -5
 RA_E_WORKSPACE = -6
 RA_MAX_PREDS = 8
+RA_MAX_PAYLOAD = 4
 RA_Q1_GROUPS = 6
 RA_LT, RA_LE, RA_GT, RA_GE, RA_EQ, RA_NE = range(6)
 OPS = {"lt": RA_LT, "le": RA_LE, "gt": RA_GT, "ge": RA_GE, "eq": RA_EQ, "ne": RA_NE}
@@ -46,6 +47,11 @@ class RAError(RuntimeError):
 
 class ra_pred(ctypes.Structure):
     _fields_ = [("op", ctypes.c_int32), ("value", ctypes.c_int32)]
+
+
+class ra_payload(ctypes.Structure):
+    _fields_ = [("col", ctypes.c_void_p), ("out", ctypes.c_void_p), ("elem_bytes", ctypes.c_int32),
+                ("_pad", ctypes.c_int32)]
 
 
 class ra_lineitem(ctypes.Structure):
@@ -113,6 +119,7 @@ _SIGS = {
     "ra_select_workspace_bytes": ([_i64, _i32, _i32], _sz),
     "ra_select": ([_vp, _i64, ra_pred, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_select_chain": ([_vp, _i64, _vp, _i32, _i32, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
+    "ra_select_rows": ([_vp, _i64, _vp, _i32, _vp, _vp, _i32, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_q1_workspace_bytes": ([_i64], _sz),
     "ra_q1": ([_vp, _i64, ctypes.c_int32, _vp, _vp, _sz, _vp], _i32),
     "ra_q1_finalize": ([_vp, _i32, _vp, _vp], _i32),
@@ -173,6 +180,12 @@ def ra_select_chain(d_in: int, n: int, h_preds, k: int, fused: int, d_out: int, 
                     d_count: int, d_ws: int, ws_bytes: int, stream: int) -> None:
     _check(_lib.ra_select_chain(d_in, n, h_preds, k, fused, d_out, out_cap, d_count, d_ws, ws_bytes,
                                 stream))
+
+
+def ra_select_rows(d_key: int, n: int, h_preds, k: int, d_rowids: int, h_payloads, m: int, out_cap: int,
+                   d_count: int, d_ws: int, ws_bytes: int, stream: int) -> None:
+    _check(_lib.ra_select_rows(d_key, n, h_preds, k, d_rowids, h_payloads, m, out_cap, d_count, d_ws, ws_bytes,
+                               stream))
 
 
 def ra_q1_workspace_bytes(n: int) -> int:

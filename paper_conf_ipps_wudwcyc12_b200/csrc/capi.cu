@@ -177,6 +177,42 @@ RA_API int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_pred
                            (cudaStream_t)stream);
 }
 
+RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_preds, int k, uint32_t* d_rowids,
+                          const ra_payload* h_payloads, int m, int64_t out_cap, int64_t* d_count, void* d_ws,
+                          size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  // d_out of the value path is unused here: pass the key as a stand-in (out_cap 0)
+  int rc = check_select_args(d_key, n, k, nullptr, 0, d_count, d_ws, ws_bytes, 1);
+  if (rc) return rc;
+  if (out_cap < 0) return fail(RA_E_INVAL, "negative out_cap");
+  if (n >= (int64_t)1 << 32) return fail(RA_E_INVAL, "n=%lld >= 2^32 (row ids are uint32)", (long long)n);
+  if (m < 0 || m > RA_MAX_PAYLOAD) return fail(RA_E_INVAL, "m=%d outside [0, %d]", m, RA_MAX_PAYLOAD);
+  if (m > 0 && !h_payloads) return fail(RA_E_INVAL, "null h_payloads with m > 0");
+  if (k > 0 && !h_preds) return fail(RA_E_INVAL, "null h_preds with k > 0");
+  for (int j = 0; j < k; ++j)
+    if (h_preds[j].op < RA_LT || h_preds[j].op > RA_NE)
+      return fail(RA_E_INVAL, "predicate %d: unknown op %d", j, (int)h_preds[j].op);
+  if ((uintptr_t)d_rowids & 3u) return fail(RA_E_INVAL, "d_rowids must be 4-byte aligned");
+  SelRows rows;
+  rows.rowids = out_cap > 0 ? d_rowids : nullptr;
+  rows.m = m;
+  for (int j = 0; j < m; ++j) {
+    const ra_payload& p = h_payloads[j];
+    if (p.elem_bytes != 4 && p.elem_bytes != 8)
+      return fail(RA_E_INVAL, "payload %d: elem_bytes %d not 4 or 8", j, (int)p.elem_bytes);
+    if ((n > 0 && !p.col) || (out_cap > 0 && !p.out)) return fail(RA_E_INVAL, "payload %d: null column", j);
+    if (((uintptr_t)p.col | (uintptr_t)p.out) & (uintptr_t)(p.elem_bytes - 1))
+      return fail(RA_E_INVAL, "payload %d: pointers not %d-byte aligned", j, (int)p.elem_bytes);
+    rows.elem_bytes[j] = p.elem_bytes;
+    rows.col[j] = p.col;
+    rows.out[j] = p.out;
+  }
+  CanonPred cp;
+  rc = canonicalize(h_preds, k, &cp);
+  if (rc) return rc;
+  return launch_select_pass(d_key, n, nullptr, cp, nullptr, out_cap, d_count, d_ws, (cudaStream_t)stream, &rows);
+}
+
 RA_API size_t ra_q1_workspace_bytes(int64_t n) {
   (void)n;
   return q1_ws_bytes();

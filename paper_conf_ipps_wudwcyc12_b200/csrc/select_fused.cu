@@ -137,6 +137,13 @@ struct SelParams {
   unsigned long long* ticket;
   uint64_t* status;  // status[tile]
   int32_t mis;       // rows of d_in's 16-B chunk before d_in (0..3)
+  // ROWS mode (tuple SELECT, ra_select_rows): the ring holds row ids; the
+  // gather writes them (rowids, nullable) and each payload field at them.
+  uint32_t* rowids;
+  int32_t m;                          // payload columns
+  int32_t pes[RA_MAX_PAYLOAD];        // element bytes (4 or 8)
+  const void* pcol[RA_MAX_PAYLOAD];   // payload columns (device)
+  void* pout[RA_MAX_PAYLOAD];         // payload outputs (device)
   int32_t lo;
   uint32_t span;  // hi - lo (the interval is never empty: see launch_select_pass)
   int32_t n_ne;
@@ -278,7 +285,10 @@ __device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams&
   return total;
 }
 
-// Compute warps: copy tile k's run of selected rows from the ring to its place.
+// Compute warps: copy tile k's run of selected rows from the ring to its place
+// (ROWS mode: the run holds row ids; write them and gather the payload
+// fields at them — the paper's gather stage, Fig 3 stage 4, L479-485).
+template <bool ROWS>
 __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k, int tid) {
   if (tid == 0) *(volatile int*)&S.demand = k;  // tell the look-back warp not to wait for later counts
   PT_BEGIN(t0);
@@ -289,11 +299,29 @@ __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k
   const int32_t* run = S.ring + S.start[k % K];  // contiguous, never wraps
   int64_t lim = P.out_cap - g;
   lim = lim < 0 ? 0 : (lim > c ? c : lim);
-  int32_t* __restrict__ out = P.out + g;
-  for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = run[e];
+  if (!ROWS) {
+    int32_t* __restrict__ out = P.out + g;
+    for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = run[e];
+    return;
+  }
+  if (P.rowids) {
+    uint32_t* __restrict__ out = P.rowids + g;
+    for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = (uint32_t)run[e];
+  }
+  for (int j = 0; j < P.m; ++j) {  // warp-uniform
+    if (P.pes[j] == 4) {
+      const int32_t* __restrict__ col = (const int32_t*)P.pcol[j];
+      int32_t* __restrict__ out = (int32_t*)P.pout[j] + g;
+      for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = __ldg(col + (uint32_t)run[e]);
+    } else {
+      const int64_t* __restrict__ col = (const int64_t*)P.pcol[j];
+      int64_t* __restrict__ out = (int64_t*)P.pout[j] + g;
+      for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = __ldg(col + (uint32_t)run[e]);
+    }
+  }
 }
 
-template <bool HAS_NE>
+template <bool HAS_NE, bool ROWS>
 __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams P) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   SelSmem& S = *reinterpret_cast<SelSmem*>(smem_raw);
@@ -539,7 +567,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         start = wp;
         break;
       }
-      write_tile(S, P, head, tid);
+      write_tile<ROWS>(S, P, head, tid);
       used -= S.cnt[head % K];
       ++head;
       forced = true;
@@ -560,12 +588,19 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
 #if RA_SEL_PTXSCATTER
         uint32_t a = ring0 + 4u * (uint32_t)p;  // byte address: one predicated store + add per row
 #pragma unroll
-        for (int c = 0; c < 4; ++c) put_if(a, fl, 1u << (4 * j + c), comp(v[j], c));
+        for (int c = 0; c < 4; ++c) {
+          // ROWS: the row id (n < 2^32 is checked by ra_select_rows)
+          const int32_t val = ROWS ? (int32_t)(uint32_t)(t * SEL_TILE + warp * WROWS - P.mis + 4 * (32 * j + lane) + c)
+                                   : comp(v[j], c);
+          put_if(a, fl, 1u << (4 * j + c), val);
+        }
 #else
         const uint32_t bits = (fl >> (4 * j)) & 0xFu;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
-          if (bits & (1u << c)) S.ring[p++] = comp(v[j], c);
+          if (bits & (1u << c))
+            S.ring[p++] = ROWS ? (int32_t)(uint32_t)(t * SEL_TILE + warp * WROWS - P.mis + 4 * (32 * j + lane) + c)
+                               : comp(v[j], c);
 #endif
         rb += (int32_t)((tot[j & 1] >> (8 * (j >> 1))) & 0xFFu);
       }
@@ -573,7 +608,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     wp = start + agg;
     // ---- gather: tile i - LAG is due
     if (i - LAG >= head) {
-      write_tile(S, P, head, tid);
+      write_tile<ROWS>(S, P, head, tid);
       used -= S.cnt[head % K];
       ++head;
     }
@@ -585,24 +620,24 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     mbar_arrive(&S.counted[i % K]);
   }
   compute_bar();  // scatters of the last tiles are visible
-  for (; head < i; ++head) write_tile(S, P, head, tid);
+  for (; head < i; ++head) write_tile<ROWS>(S, P, head, tid);
 }
 
 struct KernelCfg {
-  int grid_per_sm[64][2];
+  int grid_per_sm[64][4];
 };
 KernelCfg g_cfg;
 
-template <bool HAS_NE>
+template <bool HAS_NE, bool ROWS>
 int ensure_config(int dev, int& per_sm) {
-  int& c = g_cfg.grid_per_sm[dev][HAS_NE ? 1 : 0];
+  int& c = g_cfg.grid_per_sm[dev][(HAS_NE ? 1 : 0) + (ROWS ? 2 : 0)];
   if (!c) {
     const int smem = (int)sizeof(SelSmem);
-    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE>,
+    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE, ROWS>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(select smem)");
     int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE>, BLOCK, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE, ROWS>, BLOCK, smem);
     if (e != cudaSuccess) return cuda_fail(e, "occupancy(select)");
     if (occ < 1) return fail(RA_E_CUDA, "select kernel does not fit on an SM");
     c = occ;
@@ -628,14 +663,30 @@ int sel_ctas_per_sm() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) dev = 0;
   int per_sm = 0;
-  if (ensure_config<false>(dev, per_sm)) return -1;
+  if (ensure_config<false, false>(dev, per_sm)) return -1;
   return per_sm;
 }
 
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s) {
+                       cudaStream_t s, const SelRows* rows) {
   SelParams P;
+  P.rowids = nullptr;
+  P.m = 0;
+  for (int j = 0; j < RA_MAX_PAYLOAD; ++j) {
+    P.pes[j] = 4;
+    P.pcol[j] = nullptr;
+    P.pout[j] = nullptr;
+  }
+  if (rows) {
+    P.rowids = rows->rowids;
+    P.m = rows->m;
+    for (int j = 0; j < rows->m; ++j) {
+      P.pes[j] = rows->elem_bytes[j];
+      P.pcol[j] = rows->col[j];
+      P.pout[j] = rows->out[j];
+    }
+  }
   const uintptr_t a = (uintptr_t)d_in;
   P.mis = (int32_t)((a & 15u) >> 2);
   P.abase = (const int32_t*)(a - (a & 15u));
@@ -662,8 +713,10 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) dev = 0;
   const bool ne = P.n_ne > 0;
+  const bool rw = rows != nullptr;
   int per_sm = 1;
-  int rc = ne ? ensure_config<true>(dev, per_sm) : ensure_config<false>(dev, per_sm);
+  int rc = rw ? (ne ? ensure_config<true, true>(dev, per_sm) : ensure_config<false, true>(dev, per_sm))
+              : (ne ? ensure_config<true, false>(dev, per_sm) : ensure_config<false, false>(dev, per_sm));
   if (rc) return rc;
   const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
   int64_t grid = (int64_t)num_sms() * per_sm;
@@ -674,7 +727,8 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   const size_t smem = sizeof(SelSmem);
   void* args[] = {(void*)&P};
   cudaError_t le = cudaLaunchCooperativeKernel(
-      ne ? (const void*)select_fused_kernel<true> : (const void*)select_fused_kernel<false>,
+      rw ? (ne ? (const void*)select_fused_kernel<true, true> : (const void*)select_fused_kernel<false, true>)
+         : (ne ? (const void*)select_fused_kernel<true, false> : (const void*)select_fused_kernel<false, false>),
       dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
   if (le != cudaSuccess) return cuda_fail(le, "select_fused_kernel cooperative launch");
   count_launch();
@@ -688,7 +742,7 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
     CanonPred cp;
     int rc = canonicalize(h_preds, k, &cp);
     if (rc) return rc;
-    return launch_select_pass(d_in, n, nullptr, cp, d_out, out_cap, d_count, d_ws, s);
+    return launch_select_pass(d_in, n, nullptr, cp, d_out, out_cap, d_count, d_ws, s, nullptr);
   }
   // Unfused composition: one pass per predicate, intermediates at the end of
   // the workspace (disjoint from any status words this workspace can hold).
@@ -705,7 +759,7 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
     const bool last = (j == k - 1);
     int32_t* dst = last ? d_out : buf[j & 1];
     int64_t* dcnt = last ? d_count : &cnt[j & 1];
-    rc = launch_select_pass(src, n, src_n, cp, dst, last ? out_cap : n, dcnt, d_ws, s);
+    rc = launch_select_pass(src, n, src_n, cp, dst, last ? out_cap : n, dcnt, d_ws, s, nullptr);
     if (rc) return rc;
     src = dst;
     src_n = dcnt;

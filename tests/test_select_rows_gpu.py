@@ -1,0 +1,109 @@
+"""GPU parity of the tuple SELECT (ra_select_rows) through the
+C-ABI against the CPU oracle (oracle.select_rows): row ids and every payload
+field of the selected rows, bit-exact, in input order; Table I's SELECT and
+PROJECT examples; ragged/misaligned key views, many tiles, capacity limits."""
+import numpy as np
+import pytest
+
+import oracle
+import ragen
+from golden_io import table1_tuples
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def R():
+    import paper_conf_ipps_wudwcyc12_b200 as R
+    return R
+
+
+def check(R, key, preds, payloads, offset=0):
+    kd = torch.from_numpy(np.concatenate([np.zeros(offset, np.int32), key])).cuda()[offset:]
+    pd = [torch.from_numpy(p).cuda() for p in payloads]
+    ids, outs, cnt = R.select_rows(kd, preds, pd)
+    torch.cuda.synchronize()
+    c = int(cnt.item())
+    exp_ids, exp_outs = oracle.select_rows(key, preds, payloads)
+    assert c == exp_ids.size
+    assert np.array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
+    for o, e in zip(outs, exp_outs):
+        assert np.array_equal(o[:c].cpu().numpy(), e)
+
+
+def test_table1_examples(R):
+    cols, sel, sel_out, proj_fields, proj_out = table1_tuples()
+    f = [np.array(c, dtype=np.int32) for c in cols]
+    fd = [torch.from_numpy(c).cuda() for c in f]
+    ids, outs, cnt = R.select_rows(fd[0], [sel], fd)
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == 1 and ids[0].item() == 2
+    assert tuple(int(o[0].item()) for o in outs) == sel_out
+    ids, outs, cnt = R.select_rows(fd[0], [], [fd[j] for j in proj_fields])  # k = 0: PROJECT
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == 3
+    assert list(zip(*[o[:3].cpu().tolist() for o in outs])) == proj_out
+
+
+@pytest.mark.parametrize("n", [0, 1, 4, 8191, 8192, 8193, 3 * 8192 + 123, 1_000_003])
+@pytest.mark.parametrize("offset", [0, 1, 3])
+def test_sizes_offsets(R, n, offset):
+    key = ragen.int32_column(61 + n, n)
+    pay4 = (np.arange(n, dtype=np.int32) * 3 + 1)
+    pay8 = np.arange(n, dtype=np.int64) * (1 << 33) - 5
+    check(R, key, [("lt", 0), ("gt", -(2**30))], [pay4, pay8, key], offset)
+
+
+@pytest.mark.parametrize("s,k", [(0.0, 1), (0.01, 1), (0.5, 2), (0.9, 1), (1.0, 1)])
+def test_selectivities_many_tiles(R, s, k):
+    n = (1 << 22) + 77
+    key = ragen.int32_column(62, n)
+    preds = [("ge", -(2**31))] if s == 1.0 else [("lt", -(2**31))] if s == 0.0 else \
+        [("lt", t) for t in ragen.nested_thresholds(s, k)]
+    pay = ragen.int32_column(63, n)
+    check(R, key, preds, [pay, pay.astype(np.int64) * 11])
+
+
+def test_rowids_only_and_payload_only(R):
+    n = 500_000
+    key = ragen.int32_column(64, n)
+    kd = torch.from_numpy(key).cuda()
+    exp_ids, (exp_k,) = oracle.select_rows(key, [("lt", 12345)], [key])
+    ids, outs, cnt = R.select_rows(kd, [("lt", 12345)], [], rowids=True)
+    torch.cuda.synchronize()
+    assert np.array_equal(ids[:int(cnt.item())].cpu().numpy().astype(np.int64), exp_ids)
+    ids, outs, cnt = R.select_rows(kd, [("lt", 12345)], [kd], rowids=False)
+    torch.cuda.synchronize()
+    assert ids is None and np.array_equal(outs[0][:int(cnt.item())].cpu().numpy(), exp_k)
+    # the key gathered as a payload equals the value SELECT
+    assert np.array_equal(exp_k, oracle.select(key, [("lt", 12345)]))
+
+
+def test_capacity_truncates_but_counts(R):
+    n = 200_000
+    key = ragen.int32_column(65, n)
+    kd = torch.from_numpy(key).cuda()
+    exp_ids, _ = oracle.select_rows(key, [("lt", 0)], [])
+    cap = 1000
+    ids, outs, cnt = R.select_rows(kd, [("lt", 0)], [kd], out_cap=cap)
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == exp_ids.size
+    assert np.array_equal(ids[:cap].cpu().numpy().astype(np.int64), exp_ids[:cap])
+    assert np.array_equal(outs[0][:cap].cpu().numpy(), key[exp_ids[:cap]])
+
+
+def test_argument_errors(R):
+    kd = torch.zeros(16, dtype=torch.int32, device="cuda")
+    bad = torch.zeros(16, dtype=torch.int16, device="cuda")
+    with pytest.raises(ValueError):
+        R.select_rows(kd, [("lt", 0)], [bad])
+    pl = (R.ra_payload * 1)()
+    pl[0].col, pl[0].out, pl[0].elem_bytes = kd.data_ptr(), kd.data_ptr(), 2
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    ws = torch.zeros(1 << 20, dtype=torch.uint8, device="cuda")
+    with pytest.raises(R.RAError) as e:
+        R.ra_select_rows(kd.data_ptr(), 16, R.make_preds([("lt", 0)]), 1, 0, pl, 1, 16, cnt.data_ptr(),
+                         ws.data_ptr(), ws.numel(), 0)
+    assert e.value.code == R.RA_E_INVAL

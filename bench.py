@@ -265,6 +265,7 @@ def run_ours(args, D: Dist):
 
 
 def extras(args, D, torch, R, x, preds, kept, chain_ms):
+    s_sel = args.sel
     """Other BASELINE configs + e2e + CPU baseline, same timing rules."""
     dev = x.device
     sh = int(torch.cuda.current_stream().cuda_stream)
@@ -315,9 +316,60 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                  "fission_only": (chunk, 3, False), "fusion_fission": (chunk, 3, True)}
         ex["fission_modes"] = {m: {"ms_per_step": fission_ms(*cfg), "chunk_rows": cfg[0], "streams": cfg[1],
                                    "fused": cfg[2]} for m, cfg in modes.items()}
+        # the paper's "with round trip" (Fig 8): each SELECT copies its
+        # input to the GPU and its result back; the next SELECT starts from the host
+        if k > 1:
+            h_mid = torch.empty(n, dtype=torch.int32, pin_memory=True)
+            bufs = [h_out, h_mid]
+
+            def round_trip(i=0, kernel_done=False):
+                src, m = h_in, n
+                for j, pj in enumerate(preds):
+                    dst = bufs[j & 1]
+                    _, m = R.fission_run(src[:m], [pj], m, streams[:1], h_out=dst, h_chunk_counts=h_counts)
+                    src = dst
+                return m
+
+            assert round_trip() == kept
+            rms, _ = timed(torch, D, round_trip, 3, 1)
+            ex["fission_modes"]["with_round_trip"] = {"ms_per_step": rms, "chunk_rows": n, "streams": 1,
+                                                      "fused": False, "selects": k}
+            del h_mid
         for v in ex["fission_modes"].values():
             v["rows_per_s"] = D.world * n / (v["ms_per_step"] * 1e-3)
         del h_in, h_out, h_counts
+
+    # --- f3: tuple SELECT (Table I) on the same key column + two int32 fields,
+    # the same chain; outputs the key and both fields of the selected rows
+    f1 = torch.empty(n, dtype=torch.int32, device=dev)
+    f2 = torch.empty(n, dtype=torch.int32, device=dev)
+    ragen.int32_column_dev(CHAIN_SEED + 100, f1, stream=sh)
+    ragen.int32_column_dev(CHAIN_SEED + 101, f2, stream=sh)
+    outs = [torch.empty(n, dtype=torch.int32, device=dev) for _ in range(3)]
+    pl = (R.ra_payload * 3)()
+    for j, (c, o) in enumerate(zip((x, f1, f2), outs)):
+        pl[j].col, pl[j].out, pl[j].elem_bytes = c.data_ptr(), o.data_ptr(), 4
+    tc = torch.zeros(1, dtype=torch.int64, device=dev)
+    tws_b = R.ra_select_rows_workspace_bytes(n, k)
+    tws = torch.zeros(tws_b, dtype=torch.uint8, device=dev)
+    PT = R.make_preds(preds)
+    at = (x.data_ptr(), n, PT, k, 0, pl, 3, n, tc.data_ptr(), tws.data_ptr(), tws_b, sh)
+    tms, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_rows(*at), 20, 3)
+    tkms = tms  # select + gather kernels back to back (the whole step)
+    tk = int(tc.item())
+    assert tk == kept
+    # key read, ids written + read back, 3 fields gathered + written
+    talg = 4 * n + 2 * 4 * tk + 3 * 4 * tk + 3 * 4 * tk
+    tach = talg / (tkms * 1e-3) / 1e9
+    ex["tuple_select"] = {"rows_per_s": D.world * n / (tms * 1e-3), "ms_per_step": tms, "kernel_ms": tkms,
+                          "fields": 3, "kept": tk,
+                          "roofline": {"kernel": "select_fused_kernel<ROWS> + gather_kernel", "bound": "hbm",
+                                       "achieved": tach,
+                                       "peak": peak, "unit": "GB/s", "frac": tach / peak,
+                                       "algorithmic_bytes_per_launch": talg,
+                                       "traffic": ncu_traffic(f"select_rows_k{k}_s{s_sel}_n{n.bit_length() - 1}"),
+                                       "note": "gathers read whole 32-B sectors: DRAM traffic > algorithmic bytes"}}
+    del f1, f2, outs, tws
 
     # --- configs[0]: single SELECT on 2^20 rows, 50% (latency-bound, L2-resident)
     n1 = 1 << 20

@@ -202,11 +202,12 @@ int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h
  * SELECT over a multi-column relation.  Table I's example
  * "select [field.0==2] x -> (2,False,b)" (L153-156) returns whole tuples; in a
  * column store field 0 is the int32 key column and the other fields are
- * payload columns.  One fused pass evaluates the predicate chain on the key,
- * compacts the selected rows' ids (order-preserving) and, in the gather stage
- * (Fig 3 stage 4, L479-485), writes the ids and each payload field gathered at
- * them.  With k = 0 every row is kept: PROJECT (Table I) of the
- * payload fields.  Output = the selected tuples, stream-ordered.
+ * payload columns.  One fused pass evaluates the predicate chain on the key
+ * and compacts the selected rows' ids (order-preserving, single pass with
+ * decoupled look-back); a gather kernel on the same stream then writes each
+ * payload field at those ids (the paper's stage 4 "gather", Fig 3).
+ * With k = 0 every row is kept: PROJECT (Table I) of the payload
+ * fields.  Output = the selected tuples, stream-ordered.
  *
  *  d_key        device int32[n] (4-B aligned), n < 2^32
  *  h_preds, k   as ra_select_chain (host array, k <= RA_MAX_PREDS)
@@ -216,7 +217,7 @@ int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h
  *               naturally aligned), out device [out_cap] elements; may be
  *               NULL when m == 0
  *  d_count      device int64: number selected (the required size)
- *  d_ws         ra_select_workspace_bytes(n, k, 1) bytes, zeroed once
+ *  d_ws         ra_select_rows_workspace_bytes(n, k) bytes, zeroed once
  * Rows beyond out_cap are not written (count is still exact). */
 #define RA_MAX_PAYLOAD 4
 
@@ -226,6 +227,8 @@ typedef struct {
   int32_t elem_bytes;
   int32_t _pad;
 } ra_payload;
+
+size_t ra_select_rows_workspace_bytes(int64_t n, int k);
 
 int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_preds, int k, uint32_t* d_rowids,
                    const ra_payload* h_payloads, int m, int64_t out_cap, int64_t* d_count, void* d_ws,

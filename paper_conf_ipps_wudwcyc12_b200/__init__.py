@@ -23,7 +23,7 @@ from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, r
                   ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
                   ra_select_chain, ra_select_workspace_bytes, ra_lineitem_narrow, ra_lineitem_narrow_out,
                   ra_q1_encode, ra_q1_narrow, ra_q1_narrow_fission_run, ra_q1_narrow_fission_workspace_bytes,
-                  ra_payload, ra_select_rows)
+                  ra_payload, ra_select_rows, ra_select_rows_workspace_bytes)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
@@ -100,8 +100,8 @@ def select_rows(key, preds, payloads=(), rowids: bool = True, out_cap=None, stre
         outs.append(o)
         pl[j].col, pl[j].out, pl[j].elem_bytes = c.data_ptr(), o.data_ptr(), c.element_size()
     count = torch.empty(1, dtype=torch.int64, device=key.device)
-    need = ra_select_workspace_bytes(n, k, 1)
-    ws = workspace(key.device, "select_fused", need, stream)
+    need = ra_select_rows_workspace_bytes(n, k)
+    ws = workspace(key.device, "select_rows", need, stream)
     P = make_preds(preds)
     ra_select_rows(key.data_ptr(), n, P, k, ids.data_ptr() if ids is not None else 0, pl, len(payloads), cap,
                    count.data_ptr(), ws.data_ptr(), ws.numel(), _stream_handle(stream))

@@ -119,6 +119,7 @@ _SIGS = {
     "ra_select_workspace_bytes": ([_i64, _i32, _i32], _sz),
     "ra_select": ([_vp, _i64, ra_pred, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_select_chain": ([_vp, _i64, _vp, _i32, _i32, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
+    "ra_select_rows_workspace_bytes": ([_i64, _i32], _sz),
     "ra_select_rows": ([_vp, _i64, _vp, _i32, _vp, _vp, _i32, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_q1_workspace_bytes": ([_i64], _sz),
     "ra_q1": ([_vp, _i64, ctypes.c_int32, _vp, _vp, _sz, _vp], _i32),
@@ -180,6 +181,10 @@ def ra_select_chain(d_in: int, n: int, h_preds, k: int, fused: int, d_out: int, 
                     d_count: int, d_ws: int, ws_bytes: int, stream: int) -> None:
     _check(_lib.ra_select_chain(d_in, n, h_preds, k, fused, d_out, out_cap, d_count, d_ws, ws_bytes,
                                 stream))
+
+
+def ra_select_rows_workspace_bytes(n: int, k: int) -> int:
+    return int(_lib.ra_select_rows_workspace_bytes(n, k))
 
 
 def ra_select_rows(d_key: int, n: int, h_preds, k: int, d_rowids: int, h_payloads, m: int, out_cap: int,

@@ -177,11 +177,16 @@ RA_API int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_pred
                            (cudaStream_t)stream);
 }
 
+RA_API size_t ra_select_rows_workspace_bytes(int64_t n, int k) {
+  if (n < 0) n = 0;
+  // select status words, then a staging area for the row ids
+  return ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256 + (((size_t)n * 4 + 255) / 256) * 256;
+}
+
 RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_preds, int k, uint32_t* d_rowids,
                           const ra_payload* h_payloads, int m, int64_t out_cap, int64_t* d_count, void* d_ws,
                           size_t ws_bytes, ra_stream_t stream) {
   clear_error();
-  // d_out of the value path is unused here: pass the key as a stand-in (out_cap 0)
   int rc = check_select_args(d_key, n, k, nullptr, 0, d_count, d_ws, ws_bytes, 1);
   if (rc) return rc;
   if (out_cap < 0) return fail(RA_E_INVAL, "negative out_cap");
@@ -193,9 +198,10 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
     if (h_preds[j].op < RA_LT || h_preds[j].op > RA_NE)
       return fail(RA_E_INVAL, "predicate %d: unknown op %d", j, (int)h_preds[j].op);
   if ((uintptr_t)d_rowids & 3u) return fail(RA_E_INVAL, "d_rowids must be 4-byte aligned");
-  SelRows rows;
-  rows.rowids = out_cap > 0 ? d_rowids : nullptr;
-  rows.m = m;
+  const size_t need = ra_select_rows_workspace_bytes(n, k);
+  if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
+  GatherSpec g;
+  g.m = m;
   for (int j = 0; j < m; ++j) {
     const ra_payload& p = h_payloads[j];
     if (p.elem_bytes != 4 && p.elem_bytes != 8)
@@ -203,14 +209,21 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
     if ((n > 0 && !p.col) || (out_cap > 0 && !p.out)) return fail(RA_E_INVAL, "payload %d: null column", j);
     if (((uintptr_t)p.col | (uintptr_t)p.out) & (uintptr_t)(p.elem_bytes - 1))
       return fail(RA_E_INVAL, "payload %d: pointers not %d-byte aligned", j, (int)p.elem_bytes);
-    rows.elem_bytes[j] = p.elem_bytes;
-    rows.col[j] = p.col;
-    rows.out[j] = p.out;
+    g.elem_bytes[j] = p.elem_bytes;
+    g.col[j] = p.col;
+    g.out[j] = p.out;
   }
   CanonPred cp;
   rc = canonicalize(h_preds, k, &cp);
   if (rc) return rc;
-  return launch_select_pass(d_key, n, nullptr, cp, nullptr, out_cap, d_count, d_ws, (cudaStream_t)stream, &rows);
+  // ids go to the caller's buffer, or (payload only) to the workspace staging area
+  const size_t stage_off = ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256;
+  uint32_t* ids = d_rowids ? d_rowids : (uint32_t*)((char*)d_ws + stage_off);
+  const int64_t cap = d_rowids ? out_cap : (out_cap < n ? out_cap : n);
+  rc = launch_select_pass(d_key, n, nullptr, cp, nullptr, cap, d_count, d_ws, (cudaStream_t)stream,
+                          (cap > 0 || !d_rowids) ? ids : nullptr);
+  if (rc) return rc;
+  return launch_gather(ids, d_count, out_cap < n ? out_cap : n, g, (cudaStream_t)stream);
 }
 
 RA_API size_t ra_q1_workspace_bytes(int64_t n) {

@@ -59,21 +59,23 @@ int64_t sel_max_tiles(int64_t n);  // tiles for n rows with any 16-B misalignmen
 size_t sel_status_bytes(int64_t n);
 size_t sel_inter_bytes(int64_t n);
 
-// Tuple SELECT outputs (ra_select_rows): row ids and/or payload fields.
-struct SelRows {
-  uint32_t* rowids;
+// One select pass (one kernel).  n_max = host bound on rows; d_n (nullable) =
+// device-resident actual row count (<= n_max) produced by a previous pass.
+// rows != nullptr: row-id mode (the selected rows' ids go to rows[0..out_cap),
+// d_out unused).
+int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
+                       int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
+                       cudaStream_t s, uint32_t* rows = nullptr);
+
+// Gather of payload fields at row ids (the gather stage of a tuple SELECT):
+// out_j[i] = col_j[ids[i]] for i < min(*d_count, cap).
+struct GatherSpec {
   int m;
   int32_t elem_bytes[RA_MAX_PAYLOAD];
   const void* col[RA_MAX_PAYLOAD];
   void* out[RA_MAX_PAYLOAD];
 };
-
-// One select pass (one kernel).  n_max = host bound on rows; d_n (nullable) =
-// device-resident actual row count (<= n_max) produced by a previous pass.
-// rows != nullptr: tuple mode (d_out unused).
-int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
-                       int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, const SelRows* rows = nullptr);
+int launch_gather(const uint32_t* ids, const int64_t* d_count, int64_t cap, const GatherSpec& g, cudaStream_t s);
 
 // Fused or unfused chain (validated arguments); used by the C-ABI and fission.
 int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,

@@ -137,13 +137,7 @@ struct SelParams {
   unsigned long long* ticket;
   uint64_t* status;  // status[tile]
   int32_t mis;       // rows of d_in's 16-B chunk before d_in (0..3)
-  // ROWS mode (tuple SELECT, ra_select_rows): the ring holds row ids; the
-  // gather writes them (rowids, nullable) and each payload field at them.
-  uint32_t* rowids;
-  int32_t m;                          // payload columns
-  int32_t pes[RA_MAX_PAYLOAD];        // element bytes (4 or 8)
-  const void* pcol[RA_MAX_PAYLOAD];   // payload columns (device)
-  void* pout[RA_MAX_PAYLOAD];         // payload outputs (device)
+  uint32_t* rowids;  // ROWS mode (ra_select_rows): the ring holds row ids, written here
   int32_t lo;
   uint32_t span;  // hi - lo (the interval is never empty: see launch_select_pass)
   int32_t n_ne;
@@ -286,8 +280,7 @@ __device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams&
 }
 
 // Compute warps: copy tile k's run of selected rows from the ring to its place
-// (ROWS mode: the run holds row ids; write them and gather the payload
-// fields at them — the paper's gather stage, Fig 3 stage 4, L479-485).
+// (ROWS mode: the run holds row ids).
 template <bool ROWS>
 __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k, int tid) {
   if (tid == 0) *(volatile int*)&S.demand = k;  // tell the look-back warp not to wait for later counts
@@ -302,22 +295,9 @@ __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k
   if (!ROWS) {
     int32_t* __restrict__ out = P.out + g;
     for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = run[e];
-    return;
-  }
-  if (P.rowids) {
+  } else {
     uint32_t* __restrict__ out = P.rowids + g;
     for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = (uint32_t)run[e];
-  }
-  for (int j = 0; j < P.m; ++j) {  // warp-uniform
-    if (P.pes[j] == 4) {
-      const int32_t* __restrict__ col = (const int32_t*)P.pcol[j];
-      int32_t* __restrict__ out = (int32_t*)P.pout[j] + g;
-      for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = __ldg(col + (uint32_t)run[e]);
-    } else {
-      const int64_t* __restrict__ col = (const int64_t*)P.pcol[j];
-      int64_t* __restrict__ out = (int64_t*)P.pout[j] + g;
-      for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = __ldg(col + (uint32_t)run[e]);
-    }
   }
 }
 
@@ -669,24 +649,9 @@ int sel_ctas_per_sm() {
 
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, const SelRows* rows) {
+                       cudaStream_t s, uint32_t* rows) {
   SelParams P;
-  P.rowids = nullptr;
-  P.m = 0;
-  for (int j = 0; j < RA_MAX_PAYLOAD; ++j) {
-    P.pes[j] = 4;
-    P.pcol[j] = nullptr;
-    P.pout[j] = nullptr;
-  }
-  if (rows) {
-    P.rowids = rows->rowids;
-    P.m = rows->m;
-    for (int j = 0; j < rows->m; ++j) {
-      P.pes[j] = rows->elem_bytes[j];
-      P.pcol[j] = rows->col[j];
-      P.pout[j] = rows->out[j];
-    }
-  }
+  P.rowids = rows;
   const uintptr_t a = (uintptr_t)d_in;
   P.mis = (int32_t)((a & 15u) >> 2);
   P.abase = (const int32_t*)(a - (a & 15u));

@@ -23,6 +23,8 @@ CAPTURES = {  # report -> (summary name, traffic key, command)
     "prof_select_s01": ("select_k1_s001_n28", "select_fused_k1_s0.01_n28",
                         "python scripts/prof_driver.py select 5 28 1 0.01  (2^28 int32, k=1, s=0.01)"),
     "prof_q1": ("q1_sf10", "q1_sf10", "python scripts/prof_driver.py q1 5  (SF10, 60M rows)"),
+    "prof_rows": ("select_rows_k2_s05_n28", "select_rows_k2_s0.5_n28",
+                  "python scripts/prof_driver.py rows 5  (2^28 key + 2 int32 fields, k=2, s=0.5/stage)"),
     "prof_q1n": ("q1n_sf10", "q1n_sf10", "python scripts/prof_driver.py q1n 5  (SF10 narrow, 60M rows)"),
 }
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",

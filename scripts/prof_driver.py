@@ -1,6 +1,6 @@
 """Small driver for ncu: runs the hot-path kernels a few times at bench sizes.
 
-usage: python scripts/prof_driver.py {select|unfused|q1|q1time|select1m} [reps] [log2n] [k] [sel]
+usage: python scripts/prof_driver.py {select|unfused|rows|q1|q1n|q1time|select1m} [reps] [log2n] [k] [sel]
 """
 import os
 import sys
@@ -60,6 +60,17 @@ def main():
             print(f"q1 narrow SF{sf}: {ms:.4f} ms  {11 * n / ms / 1e6:.1f} GB/s  {n / ms * 1e3:.3e} rows/s")
             cols = enc
             torch.cuda.empty_cache()
+    elif what == "rows":  # tuple SELECT (f3): key + two int32 fields, chain k at sel
+        n = 1 << log2n
+        x = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(2, x)
+        f1 = torch.empty(n, dtype=torch.int32, device="cuda")
+        f2 = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(102, f1)
+        ragen.int32_column_dev(103, f2)
+        preds = [("lt", t) for t in ragen.nested_thresholds(sel, k)]
+        for _ in range(reps):
+            R.select_rows(x, preds, [x, f1, f2], rowids=False)
     elif what == "q1n":  # narrow Q1 at SF10 (for ncu)
         n = ragen.rows_for_sf(10)
         cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")

@@ -61,6 +61,8 @@ def lib() -> ctypes.CDLL:
             f.restype = i64
         L.oracle_select_chunked.argtypes = [vp, i64, vp, i32, i64, vp]
         L.oracle_select_chunked.restype = i64
+        L.oracle_select_multi.argtypes = [vp, i64, vp, vp, vp, i32, vp, vp]
+        L.oracle_select_multi.restype = i32
         L.oracle_select_rows.argtypes = [vp, i64, vp, i32, i32, vp, vp, vp, vp]
         L.oracle_select_rows.restype = i64
         L.oracle_q1.argtypes = [vp, vp, vp, vp, vp, vp, vp, i64, ctypes.c_int32, vp, vp]
@@ -114,6 +116,25 @@ def select_chunked(x, preds, chunk: int) -> np.ndarray:
     if m < 0:
         raise ValueError(f"oracle_select_chunked failed ({m})")
     return out[:m].copy()
+
+
+def select_multi(x, chains):
+    """Several SELECTs on the same input (Fig 2(c)): one order-preserving
+    output per predicate chain in ``chains``."""
+    x = _as_i32(x)
+    flat = [p for c in chains for p in c]
+    P = _preds(flat)
+    M = len(chains)
+    off = (ctypes.c_int32 * max(1, M))(*[sum(len(c) for c in chains[:o]) for o in range(M)])
+    ks = (ctypes.c_int32 * max(1, M))(*[len(c) for c in chains])
+    outs = [np.empty(max(1, x.size), dtype=np.int32) for _ in range(M)]
+    op = (ctypes.c_void_p * max(1, M))(*[o.ctypes.data for o in outs])
+    counts = np.zeros(max(1, M), dtype=np.int64)
+    rc = lib().oracle_select_multi(x.ctypes.data, x.size, ctypes.addressof(P), ctypes.addressof(off),
+                                   ctypes.addressof(ks), M, ctypes.addressof(op), counts.ctypes.data)
+    if rc < 0:
+        raise ValueError(f"oracle_select_multi failed ({rc})")
+    return [o[:c].copy() for o, c in zip(outs, counts[:M])]
 
 
 def select_rows(key, preds, payloads=()):

@@ -114,6 +114,33 @@ ORACLE_API int64_t oracle_select_chunked(const int32_t* x, int64_t n, const orac
   return total;
 }
 
+/* Several SELECTs filtering the same input (Fig 2(c): "different
+ * SELECT operators need to filter the same input data"): output o is the
+ * order-preserving SELECT of x by its own chain P[off[o] .. off[o]+k[o]),
+ * exactly as oracle_select would give it; counts[o] receives its size.  One
+ * pass over x (each element tested against every chain).  Returns 0, or -1
+ * for an invalid predicate. */
+ORACLE_API int oracle_select_multi(const int32_t* x, int64_t n, const oracle_pred* P, const int32_t* off,
+                                   const int32_t* k, int M, int32_t* const* outs, int64_t* counts) {
+  for (int o = 0; o < M; ++o) {
+    counts[o] = 0;
+    for (int j = 0; j < k[o]; ++j)
+      if (oracle_cmp(P[off[o] + j].op, 0, P[off[o] + j].value) < 0) return -1;
+  }
+  for (int64_t i = 0; i < n; ++i) {
+    for (int o = 0; o < M; ++o) {
+      int keep = 1;
+      for (int j = 0; j < k[o]; ++j)
+        if (!oracle_cmp(P[off[o] + j].op, x[i], P[off[o] + j].value)) keep = 0;
+      if (keep) {
+        if (outs && outs[o]) outs[o][counts[o]] = x[i];
+        counts[o]++;
+      }
+    }
+  }
+  return 0;
+}
+
 /* SELECT over a multi-column relation (Table I: "select
  * [field.0==2] x -> (2,False,b)" returns whole tuples; the first field is the
  * key).  Column store: `key` is field 0, cols[0..m) are further fields of

@@ -132,3 +132,23 @@ def test_select_rows_matches_numpy_and_value_select():
     assert np.array_equal(rowids, np.flatnonzero(mask))
     assert np.array_equal(okey, x[mask]) and np.array_equal(opay, pay[mask])
     assert np.array_equal(okey, oracle.select(x, preds))
+
+
+# ----------------------------------------------------- several SELECTs (f2)
+@settings(max_examples=200, deadline=None)
+@given(xs=st.lists(st.one_of(I32, st.integers(-5, 5)), max_size=60),
+       chains=st.lists(st.lists(st.tuples(st.sampled_from(OPS), st.one_of(I32, st.integers(-5, 5))), max_size=4),
+                       min_size=1, max_size=4))
+def test_select_multi_equals_brute_force_per_output(xs, chains):
+    outs = oracle.select_multi(xs, chains)
+    assert [o.tolist() for o in outs] == [brute(xs, c) for c in chains]
+
+
+def test_select_multi_numpy_and_disjoint_cover():
+    """Two complementary SELECTs (x < t, x >= t) partition the input: the
+    outputs' sizes add to n, and each equals numpy boolean indexing."""
+    x = ragen.int32_column(10, 200_001)
+    t = int(x[123])
+    lo, hi = oracle.select_multi(x, [[("lt", t)], [("ge", t)]])
+    assert np.array_equal(lo, x[x < t]) and np.array_equal(hi, x[x >= t])
+    assert lo.size + hi.size == x.size

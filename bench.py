@@ -339,6 +339,41 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
             v["rows_per_s"] = D.world * n / (v["ms_per_step"] * 1e-3)
         del h_in, h_out, h_counts
 
+    # --- f2: two SELECTs filtering the same input (Fig 2(c)): one fused pass
+    # vs the two SELECT kernels run one after the other (two input reads)
+    chains = [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)]]
+    mo = [torch.empty(n, dtype=torch.int32, device=dev) for _ in range(2)]
+    mc = torch.zeros(2, dtype=torch.int64, device=dev)
+    mws_b = R.ra_select_workspace_bytes(n, R.RA_MAX_PREDS, 1)
+    mws = torch.zeros(mws_b, dtype=torch.uint8, device=dev)
+    keepP = [R.make_preds(c) for c in chains]
+    mch = (ctypes.c_void_p * 2)(*[ctypes.addressof(p_) for p_ in keepP])
+    mks = (ctypes.c_int * 2)(*[len(c) for c in chains])
+    mop = (ctypes.c_void_p * 2)(*[o.data_ptr() for o in mo])
+    mcap = (ctypes.c_int64 * 2)(n, n)
+    mcp = (ctypes.c_void_p * 2)(mc.data_ptr(), mc.data_ptr() + 8)
+    am = (x.data_ptr(), n, mch, mks, 2, mop, mcap, mcp, mws.data_ptr(), mws_b, sh)
+    mms, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_multi(*am), 20, 3)
+    c0, c1 = (int(v) for v in mc.cpu().tolist())
+    sep = [(x.data_ptr(), n, keepP[o], len(chains[o]), 1, mo[o].data_ptr(), n, mc.data_ptr() + 8 * o,
+            mws.data_ptr(), mws_b, sh) for o in range(2)]
+
+    def two_kernels(i=0, kernel_done=False):
+        R.ra_select_chain(*sep[0])
+        R.ra_select_chain(*sep[1])
+    sms, _ = timed(torch, D, two_kernels, 20, 3)
+    assert [int(v) for v in mc.cpu().tolist()] == [c0, c1]
+    malg = 4 * n + 4 * (c0 + c1)
+    mach = malg / (mms * 1e-3) / 1e9
+    ex["select_multi"] = {"outputs": 2, "chains": [[list(p_) for p_ in c] for c in chains], "kept": [c0, c1],
+                          "rows_per_s": D.world * n / (mms * 1e-3), "ms_per_step": mms,
+                          "two_separate_selects_ms": sms, "fused_over_separate": sms / mms,
+                          "bytes_ratio": (8 * n + 4 * (c0 + c1)) / malg,
+                          "roofline": {"kernel": "select_fused_kernel<M=2>", "bound": "hbm", "achieved": mach,
+                                       "peak": peak, "unit": "GB/s", "frac": mach / peak,
+                                       "algorithmic_bytes_per_launch": malg}}
+    del mo, mws
+
     # --- f3: tuple SELECT (Table I) on the same key column + two int32 fields,
     # the same chain; outputs the key and both fields of the selected rows
     f1 = torch.empty(n, dtype=torch.int32, device=dev)

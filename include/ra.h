@@ -198,6 +198,27 @@ int ra_q1(const ra_lineitem* h_cols, int64_t n, int32_t shipdate_cutoff,
 int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h_rows,
                    int* n_rows);
 
+/* ============================================================ SEVERAL SELECTs
+ * Several SELECT operators filtering the same input (Fig 2(c)
+ * L286-288, "different SELECT operators need to filter the same input data").
+ * One fused pass reads the input once, evaluates every output's predicate
+ * chain in registers and compacts each output separately (order-preserving;
+ * both tile aggregates travel in one look-back status word).  Output o equals
+ * ra_select_chain(d_in, chains[o]).  Stream-ordered.
+ *
+ *  d_in          device int32[n] (4-B aligned)
+ *  h_chains[o]   host array of ks[o] predicates (0 <= ks[o] <= RA_MAX_PREDS)
+ *  M             number of outputs, 1 <= M <= RA_MAX_OUTPUTS
+ *  d_outs[o]     device int32[out_caps[o]]
+ *  d_counts[o]   device int64: output o's size (the required size)
+ *  d_ws          ra_select_workspace_bytes(n, RA_MAX_PREDS, 1), zeroed once
+ * Rows beyond out_caps[o] are not written (the count is still exact). */
+#define RA_MAX_OUTPUTS 2
+
+int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const* h_chains, const int* ks, int M,
+                    int32_t* const* d_outs, const int64_t* out_caps, int64_t* const* d_counts, void* d_ws,
+                    size_t ws_bytes, ra_stream_t stream);
+
 /* ============================================================ TUPLE SELECT
  * SELECT over a multi-column relation.  Table I's example
  * "select [field.0==2] x -> (2,False,b)" (L153-156) returns whole tuples; in a

@@ -23,7 +23,7 @@ from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, r
                   ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
                   ra_select_chain, ra_select_workspace_bytes, ra_lineitem_narrow, ra_lineitem_narrow_out,
                   ra_q1_encode, ra_q1_narrow, ra_q1_narrow_fission_run, ra_q1_narrow_fission_workspace_bytes,
-                  ra_payload, ra_select_rows, ra_select_rows_workspace_bytes)
+                  ra_payload, ra_select_rows, ra_select_rows_workspace_bytes, ra_select_multi, RA_MAX_PREDS)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
@@ -77,6 +77,30 @@ def select_chain(x, preds, fused: bool = True, out=None, count=None, stream=None
     ra_select_chain(x.data_ptr(), n, P, k, int(fused), out.data_ptr(), out.numel(), count.data_ptr(),
                     ws.data_ptr(), ws.numel(), _stream_handle(stream))
     return out, count
+
+
+def select_multi(x, chains, outs=None, stream=None):
+    """Several SELECTs on the same CUDA int32 tensor in one pass (Fig 2(c)).
+
+    ``chains``: list of 1..RA_MAX_OUTPUTS predicate chains.  Returns
+    ``(outs, counts)``: ``outs[o][:counts[o]]`` is chain o's selection in
+    input order; ``counts`` a CUDA int64 tensor (not synchronised)."""
+    torch = _torch()
+    if not (x.is_cuda and x.dtype == torch.int32 and x.is_contiguous()):
+        raise ValueError("x must be a contiguous CUDA int32 tensor")
+    n, M = x.numel(), len(chains)
+    if outs is None:
+        outs = [torch.empty(max(1, n), dtype=torch.int32, device=x.device) for _ in range(M)]
+    counts = torch.empty(max(1, M), dtype=torch.int64, device=x.device)
+    keep = [make_preds(c) for c in chains]
+    ch = (ctypes.c_void_p * M)(*[ctypes.addressof(p) for p in keep])
+    ks = (ctypes.c_int * M)(*[len(c) for c in chains])
+    op = (ctypes.c_void_p * M)(*[o.data_ptr() for o in outs])
+    caps = (ctypes.c_int64 * M)(*[o.numel() for o in outs])
+    cp = (ctypes.c_void_p * M)(*[counts.data_ptr() + 8 * o for o in range(M)])
+    ws = workspace(x.device, "select_fused", ra_select_workspace_bytes(n, RA_MAX_PREDS, 1), stream)
+    ra_select_multi(x.data_ptr(), n, ch, ks, M, op, caps, cp, ws.data_ptr(), ws.numel(), _stream_handle(stream))
+    return outs, counts
 
 
 def select_rows(key, preds, payloads=(), rowids: bool = True, out_cap=None, stream=None):

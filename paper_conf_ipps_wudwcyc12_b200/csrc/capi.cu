@@ -177,6 +177,35 @@ RA_API int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_pred
                            (cudaStream_t)stream);
 }
 
+RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const* h_chains, const int* ks, int M,
+                           int32_t* const* d_outs, const int64_t* out_caps, int64_t* const* d_counts, void* d_ws,
+                           size_t ws_bytes, ra_stream_t stream) {
+  clear_error();
+  if (M < 1 || M > RA_MAX_OUTPUTS) return fail(RA_E_INVAL, "M=%d outside [1, %d]", M, RA_MAX_OUTPUTS);
+  if (!h_chains || !ks || !d_outs || !out_caps || !d_counts) return fail(RA_E_INVAL, "null argument");
+  CanonPred cp[RA_MAX_OUTPUTS];
+  for (int o = 0; o < M; ++o) {
+    int rc = check_select_args(d_in, n, ks[o], d_outs[o], out_caps[o], d_counts[o], d_ws, ws_bytes, 1);
+    if (rc) return rc;
+    if (ks[o] > 0 && !h_chains[o]) return fail(RA_E_INVAL, "null chain %d with k > 0", o);
+    for (int j = 0; j < ks[o]; ++j)
+      if (h_chains[o][j].op < RA_LT || h_chains[o][j].op > RA_NE)
+        return fail(RA_E_INVAL, "output %d predicate %d: unknown op %d", o, j, (int)h_chains[o][j].op);
+    rc = canonicalize(h_chains[o], ks[o], &cp[o]);
+    if (rc) return rc;
+  }
+  if (M == 1)
+    return launch_select_pass(d_in, n, nullptr, cp[0], d_outs[0], out_caps[0], d_counts[0], d_ws,
+                              (cudaStream_t)stream);
+  SelSecond second;
+  second.cp = cp[1];
+  second.out = d_outs[1];
+  second.out_cap = out_caps[1];
+  second.d_count = d_counts[1];
+  return launch_select_pass(d_in, n, nullptr, cp[0], d_outs[0], out_caps[0], d_counts[0], d_ws, (cudaStream_t)stream,
+                            nullptr, &second);
+}
+
 RA_API size_t ra_select_rows_workspace_bytes(int64_t n, int k) {
   if (n < 0) n = 0;
   // select status words, then a staging area for the row ids

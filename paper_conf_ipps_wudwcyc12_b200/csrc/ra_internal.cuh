@@ -63,9 +63,16 @@ size_t sel_inter_bytes(int64_t n);
 // device-resident actual row count (<= n_max) produced by a previous pass.
 // rows != nullptr: row-id mode (the selected rows' ids go to rows[0..out_cap),
 // d_out unused).
+// second != nullptr: a second predicate / output in the same pass (ra_select_multi).
+struct SelSecond {
+  CanonPred cp;
+  int32_t* out;
+  int64_t out_cap;
+  int64_t* d_count;
+};
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, uint32_t* rows = nullptr);
+                       cudaStream_t s, uint32_t* rows = nullptr, const SelSecond* second = nullptr);
 
 // Gather of payload fields at row ids (the gather stage of a tuple SELECT):
 // out_j[i] = col_j[ids[i]] for i < min(*d_count, cap).

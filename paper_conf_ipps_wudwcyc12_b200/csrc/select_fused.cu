@@ -60,6 +60,8 @@
 
 #include <stdio.h>
 
+#include <type_traits>
+
 #include "ra_internal.cuh"
 
 namespace ra {
@@ -124,7 +126,7 @@ constexpr int NPK = SEL_VEC / 4;         // packed count words per lane (4 rows 
 static_assert(SEL_VEC == 8, "per-j counts are packed as 2 words x 4 bytes; fl has 32 bits");
 static_assert(NW <= 32, "one warp reduces the per-warp counts");
 static_assert(LAG >= D2 + 1, "a tile is placed before it is due");
-static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");
+static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");  // (M == 2: 2 x SEL_TILE, SelSmem2)
 
 struct SelParams {
   const int32_t* abase;  // 16-B aligned base, = d_in - mis
@@ -138,15 +140,25 @@ struct SelParams {
   uint64_t* status;  // status[tile]
   int32_t mis;       // rows of d_in's 16-B chunk before d_in (0..3)
   uint32_t* rowids;  // ROWS mode (ra_select_rows): the ring holds row ids, written here
+  // M == 2 (ra_select_multi): a second predicate and output on the same input
+  int32_t lo2;
+  uint32_t span2;
+  int32_t n_ne2;
+  int32_t ne2[RA_MAX_PREDS];
+  int32_t* out2;
+  int64_t out_cap2;
+  int64_t* d_count2;
   int32_t lo;
   uint32_t span;  // hi - lo (the interval is never empty: see launch_select_pass)
   int32_t n_ne;
   int32_t ne[RA_MAX_PREDS];
 };
 
-struct __align__(128) SelSmem {
+template <int RING>
+struct __align__(128) SelSmemT {
+  static constexpr int kRing = RING;
   int4 in[SEL_INSLOTS][SEL_TILE / 4];  // input tiles (bulk-copy destination)
-  int32_t ring[SEL_OUTRING];           // selected rows of counted, not yet written tiles
+  int32_t ring[RING];                  // selected rows of counted, not yet written tiles
   uint64_t win[Q][WIN_WORDS];          // look-back windows (bulk-copied status words)
   uint64_t full[SEL_INSLOTS];          // TMA -> compute: tile landed (or end marker)
   uint64_t empty[SEL_INSLOTS];         // compute -> producer: slot read
@@ -157,13 +169,22 @@ struct __align__(128) SelSmem {
   int64_t tidx[K];                     // tile index of CTA-local tile k (-1: no more tiles)
   int64_t wlo[Q], whi[Q];              // window bounds [lo, hi) of each window slot
   int64_t goff[K];                     // tile output offsets
-  uint32_t wtot[2][NW];                // per-warp selected counts (double-buffered by tile)
+  uint32_t wtot[2][2][NW];             // [tile parity][output][warp] selected counts
   int32_t cnt[K];                      // tile aggregates
+  int32_t cnt2[K];                     // M == 2: second output's tile aggregates (run after the first)
+  int64_t goff2[K];                    // M == 2: second output's tile offsets
   int32_t start[K];                    // tile run start in the ring
   int64_t n;
   uint32_t epoch;
   int32_t demand;  // oldest tile the compute warps are waiting to write (-1: none yet)
 };
+// One output: a 40 KB ring (2 CTAs/SM).  Two outputs (ra_select_multi): a
+// tile's two runs together hold up to 2 x 8192 rows, so the ring doubles
+// (1 CTA/SM).
+using SelSmem = SelSmemT<SEL_OUTRING>;
+using SelSmem2 = SelSmemT<2 * SEL_TILE>;
+template <int M>
+using SmemFor = typename std::conditional<M == 2, SelSmem2, SelSmem>::type;
 
 using dev::smem_u32;
 using dev::mbar_init;
@@ -197,6 +218,17 @@ __device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
   return k;
 }
 
+template <bool HAS_NE>
+__device__ __forceinline__ bool keep2(int32_t x, const SelParams& P) {
+  bool k = (uint32_t)(x - P.lo2) <= P.span2;
+  if (HAS_NE) {
+#pragma unroll
+    for (int j = 0; j < RA_MAX_PREDS; ++j)
+      if (j < P.n_ne2) k &= (x != P.ne2[j]);
+  }
+  return k;
+}
+
 __device__ __forceinline__ int32_t comp(const int4& v, int c) {
   return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
 }
@@ -215,7 +247,8 @@ __device__ __forceinline__ void put_if(uint32_t& a, uint32_t fl, uint32_t mask, 
 }
 
 // Issue the bulk copy of tile t into input slot s (one thread).
-__device__ __forceinline__ void issue_tile(SelSmem& S, const SelParams& P, int64_t nv, int64_t t, int s) {
+template <typename SM>
+__device__ __forceinline__ void issue_tile(SM& S, const SelParams& P, int64_t nv, int64_t t, int s) {
   const int64_t v0 = t * SEL_TILE;
   int64_t rows = nv - v0;
   if (rows > SEL_TILE) rows = SEL_TILE;
@@ -228,7 +261,8 @@ __device__ __forceinline__ void issue_tile(SelSmem& S, const SelParams& P, int64
 // Look-back warp, lane 0: bulk-copy window [lo, hi) of status words into slot
 // q (16-B aligned start: one extra word may precede lo).  A window longer than
 // the slot (a CTA that ran slow) is not copied; it is read directly instead.
-__device__ __forceinline__ void issue_window(SelSmem& S, const SelParams& P, int64_t lo, int64_t hi, int q) {
+template <typename SM>
+__device__ __forceinline__ void issue_window(SM& S, const SelParams& P, int64_t lo, int64_t hi, int q) {
   S.wlo[q] = lo;
   S.whi[q] = hi;
   const int64_t s0 = lo & ~1ll;
@@ -248,7 +282,8 @@ __device__ __forceinline__ void issue_window(SelSmem& S, const SelParams& P, int
 // <= SEL_TILE < 2^32, so a word published by this launch has its high half
 // exactly `want` = (FLAG_A | tag) >> 32: readiness is one compare and each
 // pass sums in 32 bits (one REDUX).  Words still unpublished are re-polled.
-__device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams& P, int q, int lane, uint32_t want) {
+template <typename SM>
+__device__ __forceinline__ int64_t window_sum(const SM& S, const SelParams& P, int q, int lane, uint32_t want) {
   const int64_t lo = S.wlo[q], hi = S.whi[q];
   const int64_t s0 = lo & ~1ll;
   const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
@@ -279,10 +314,47 @@ __device__ __forceinline__ int64_t window_sum(const SelSmem& S, const SelParams&
   return total;
 }
 
+// M == 2: the status word carries both outputs' aggregates (16 bits each in
+// the low word); sum them separately.  Same readiness rule as window_sum.
+template <typename SM>
+__device__ __forceinline__ void window_sum2(const SM& S, const SelParams& P, int q, int lane, uint32_t want,
+                                            int64_t& t0, int64_t& t1) {
+  const int64_t lo = S.wlo[q], hi = S.whi[q];
+  const int64_t s0 = lo & ~1ll;
+  const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
+  t0 = t1 = 0;
+  for (int64_t base = lo; base < hi; base += PASS_WORDS) {
+    uint64_t w[LBW];
+#pragma unroll
+    for (int c = 0; c < LBW; ++c) {
+      const int64_t idx = base + LBW * lane + c;
+      w[c] = idx >= hi ? ((uint64_t)want << 32) : copied ? S.win[q][idx - s0] : dev::ld_relaxed_u64(P.status + idx);
+    }
+    for (int spins = 0;; ++spins) {
+      bool missing = false;
+#pragma unroll
+      for (int c = 0; c < LBW; ++c) missing |= (uint32_t)(w[c] >> 32) != want;
+      if (!__any_sync(0xffffffffu, missing)) break;
+      if (spins > 1) __nanosleep(64);
+#pragma unroll
+      for (int c = 0; c < LBW; ++c)
+        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + LBW * lane + c);
+    }
+    uint32_t v0 = 0, v1 = 0;
+#pragma unroll
+    for (int c = 0; c < LBW; ++c) {
+      v0 += (uint32_t)w[c] & 0xFFFFu;
+      v1 += ((uint32_t)w[c] >> 16) & 0xFFFFu;
+    }
+    t0 += __reduce_add_sync(0xffffffffu, v0);
+    t1 += __reduce_add_sync(0xffffffffu, v1);
+  }
+}
+
 // Compute warps: copy tile k's run of selected rows from the ring to its place
 // (ROWS mode: the run holds row ids).
-template <bool ROWS>
-__device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k, int tid) {
+template <bool ROWS, int M, typename SM>
+__device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int tid) {
   if (tid == 0) *(volatile int*)&S.demand = k;  // tell the look-back warp not to wait for later counts
   PT_BEGIN(t0);
   mbar_wait(&S.placed[k % K], (uint32_t)((k / K) & 1));
@@ -292,6 +364,14 @@ __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k
   const int32_t* run = S.ring + S.start[k % K];  // contiguous, never wraps
   int64_t lim = P.out_cap - g;
   lim = lim < 0 ? 0 : (lim > c ? c : lim);
+  if (M == 2) {  // the second output's run follows the first in the ring
+    const int64_t g2 = S.goff2[k % K];
+    const int32_t c2 = S.cnt2[k % K];
+    int64_t lim2 = P.out_cap2 - g2;
+    lim2 = lim2 < 0 ? 0 : (lim2 > c2 ? c2 : lim2);
+    int32_t* __restrict__ out2 = P.out2 + g2;
+    for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = run[c + e];
+  }
   if (!ROWS) {
     int32_t* __restrict__ out = P.out + g;
     for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = run[e];
@@ -301,10 +381,13 @@ __device__ __forceinline__ void write_tile(SelSmem& S, const SelParams& P, int k
   }
 }
 
-template <bool HAS_NE, bool ROWS>
+template <bool HAS_NE, bool ROWS, int M>
 __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams P) {
+  static_assert(M == 1 || (M == 2 && !ROWS), "two outputs in value mode only");
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  SelSmem& S = *reinterpret_cast<SelSmem*>(smem_raw);
+  using SM = SmemFor<M>;
+  constexpr int RING = SM::kRing;
+  SM& S = *reinterpret_cast<SM*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
   if (tid == 0) {
@@ -374,6 +457,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ======================= look-back warp: tile offsets =======================
     const uint32_t want = (uint32_t)((FLAG_A | (tag << TAG_SHIFT)) >> 32);
     int64_t my_prefix = 0;  // inclusive prefix of this CTA's last placed tile
+    int64_t my_prefix2 = 0;  // M == 2: the same for the second output
     int64_t t_last = -1;    // tile index of the last window copied
     int m = 0x7fffffff;     // tiles of this CTA, known once the end marker is counted
     // Decisions are warp-uniform: a lane that sees a barrier phase complete has
@@ -420,14 +504,25 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         mbar_wait(&S.winfull[q], (uint32_t)((k / Q) & 1));
         PT_END(6, t0, lane == 0);
         PT_BEGIN(t1);
-        const int64_t g = my_prefix + window_sum(S, P, q, lane, want);
+        int64_t g, g2 = 0;
+        if constexpr (M == 2) {
+          int64_t w0, w1;
+          window_sum2(S, P, q, lane, want, w0, w1);
+          g = my_prefix + w0;
+          g2 = my_prefix2 + w1;
+          my_prefix2 = g2 + S.cnt2[k % K];
+        } else {
+          g = my_prefix + window_sum(S, P, q, lane, want);
+        }
         PT_END(7, t1, lane == 0);
         const int64_t tp = S.whi[q];
         my_prefix = g + S.cnt[k % K];
         if (lane == 0) {
           S.goff[k % K] = g;
+          if (M == 2) S.goff2[k % K] = g2;
           if (tp == ntiles - 1) {  // every tile has published (read the epoch): advance it
             *P.d_count = my_prefix;
+            if (M == 2) *P.d_count2 = my_prefix2;
             st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
           }
           mbar_arrive(&S.placed[k % K]);
@@ -441,7 +536,10 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       if (atomicAdd(&P.hdr[H_DONE], 1u) == gridDim.x - 1) {
         *P.ticket = 0ull;
         P.hdr[H_DONE] = 0u;
-        if (ntiles == 0) *P.d_count = 0;
+        if (ntiles == 0) {
+          *P.d_count = 0;
+          if (M == 2) *P.d_count2 = 0;
+        }
       }
     }
     return;
@@ -469,61 +567,84 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       for (int j = 0; j < SEL_VEC; ++j) v[j] = base[32 * j + lane];
     }
     const int64_t v0 = t * SEL_TILE + warp * WROWS;
-    uint32_t fl = 0;  // bit 4j+c: row warp*1024 + 4*(32j + lane) + c selected
+    uint32_t fl = 0;   // bit 4j+c: row warp*1024 + 4*(32j + lane) + c selected
+    uint32_t fl2 = 0;  // M == 2: the same for the second output
     if (v0 >= P.mis && v0 + WROWS <= nv) {
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) fl |= (uint32_t)keep<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
+        for (int c = 0; c < 4; ++c) {
+          fl |= (uint32_t)keep<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
+          if (M == 2) fl2 |= (uint32_t)keep2<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
+        }
     } else {
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
         const int64_t e0 = v0 + 4 * (32 * j + lane);
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
-          const bool k = keep<HAS_NE>(comp(v[j], c), P) & (e0 + c >= P.mis) & (e0 + c < nv);
-          fl |= (uint32_t)k << (4 * j + c);
+          const bool in = (e0 + c >= P.mis) & (e0 + c < nv);
+          fl |= (uint32_t)(keep<HAS_NE>(comp(v[j], c), P) & in) << (4 * j + c);
+          if (M == 2) fl2 |= (uint32_t)(keep2<HAS_NE>(comp(v[j], c), P) & in) << (4 * j + c);
         }
       }
     }
     // ---- buffer: order (warp, j, lane, c); packed per-j counts, warp scans.
     // SWAR popcount of each nibble of fl (nibble j = the lane's 4 rows of
     // vector j), then j goes to word j&1, byte j>>1 (8 bits: a warp total <= 128).
-    uint32_t packed[NPK], inc[NPK], tot[NPK];
-    {
-      uint32_t x = fl - ((fl >> 1) & 0x55555555u);
+    // M == 2: words NPK.. hold the second output's counts.
+    constexpr int NQ = NPK * M;
+    uint32_t packed[NQ], inc[NQ], tot[NQ];
+#pragma unroll
+    for (int o = 0; o < M; ++o) {
+      const uint32_t f = o == 0 ? fl : fl2;
+      uint32_t x = f - ((f >> 1) & 0x55555555u);
       x = (x & 0x33333333u) + ((x >> 2) & 0x33333333u);
-      packed[0] = x & 0x0F0F0F0Fu;
-      packed[1] = (x >> 4) & 0x0F0F0F0Fu;
-      inc[0] = packed[0];
-      inc[1] = packed[1];
+      packed[NPK * o] = x & 0x0F0F0F0Fu;
+      packed[NPK * o + 1] = (x >> 4) & 0x0F0F0F0Fu;
+      inc[NPK * o] = packed[NPK * o];
+      inc[NPK * o + 1] = packed[NPK * o + 1];
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
 #pragma unroll
-      for (int q = 0; q < NPK; ++q) {
+      for (int q = 0; q < NQ; ++q) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, inc[q], d);
         if (lane >= d) inc[q] += y;
       }
     }
-    uint32_t wtotal = 0;
+    uint32_t wtotal[M];
 #pragma unroll
-    for (int q = 0; q < NPK; ++q) {
+    for (int o = 0; o < M; ++o) wtotal[o] = 0;
+#pragma unroll
+    for (int q = 0; q < NQ; ++q) {
       tot[q] = __shfl_sync(0xffffffffu, inc[q], 31);  // per-row warp totals (<= 128 each)
-      wtotal += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
+      wtotal[q / NPK] += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
     }
-    if (lane == 0) S.wtot[i & 1][warp] = wtotal;
+    if (lane == 0) {
+#pragma unroll
+      for (int o = 0; o < M; ++o) S.wtot[i & 1][o][warp] = wtotal[o];
+    }
     PT_BEGIN(tb);
     compute_bar();  // B1: wtot visible; every warp is done with this tile's input slot
     PT_END(3, tb, tid == 0);
     PT_END(13, tb, tid == 224);
-    const uint32_t wt = lane < NW ? S.wtot[i & 1][lane] : 0u;
+    const uint32_t wt = lane < NW ? S.wtot[i & 1][0][lane] : 0u;
     const int32_t agg = (int32_t)__reduce_add_sync(0xffffffffu, wt);
     const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
+    int32_t agg2 = 0, wbase2 = 0;
+    if (M == 2) {
+      const uint32_t wt2 = lane < NW ? S.wtot[i & 1][1][lane] : 0u;
+      agg2 = (int32_t)__reduce_add_sync(0xffffffffu, wt2);
+      wbase2 = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt2 : 0u);
+    }
+    const int32_t rows_in = agg + agg2;  // ring rows this tile needs (both runs)
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
       mbar_arrive(&S.empty[slot]);  // input slot free: the producer refills it
-      dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
+      const uint64_t aggw = M == 2 ? ((uint64_t)agg | ((uint64_t)agg2 << 16)) : (uint64_t)agg;
+      dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | aggw);
       S.cnt[i % K] = agg;
+      if (M == 2) S.cnt2[i % K] = agg2;
       S.tidx[i % K] = t;
       mbar_arrive(&S.counted[i % K]);
     }
@@ -541,29 +662,32 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       const int32_t rp = S.start[head % K];
       const bool wrapped = rp > wp || (rp == wp && used > 0);
       if (!wrapped) {
-        if (wp + agg <= SEL_OUTRING) { start = wp; break; }
-        if (agg <= rp) { start = 0; break; }
-      } else if (wp + agg <= rp) {
+        if (wp + rows_in <= RING) { start = wp; break; }
+        if (rows_in <= rp) { start = 0; break; }
+      } else if (wp + rows_in <= rp) {
         start = wp;
         break;
       }
-      write_tile<ROWS>(S, P, head, tid);
-      used -= S.cnt[head % K];
+      write_tile<ROWS, M, SM>(S, P, head, tid);
+      used -= S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0);
       ++head;
       forced = true;
     }
     if (forced) compute_bar();  // rows written out are read before they are overwritten
     if (tid == 0) S.start[i % K] = start;
-    used += agg;
-    // ---- scatter the tile into the ring
-    {
-      int32_t rb = start + wbase;
+    used += rows_in;
+    // ---- scatter the tile into the ring (M == 2: the second run after the first)
+#pragma unroll
+    for (int o = 0; o < M; ++o) {
+      const uint32_t f = o == 0 ? fl : fl2;
+      int32_t rb = start + (o == 0 ? wbase : agg + wbase2);
 #if RA_SEL_PTXSCATTER
       const uint32_t ring0 = smem_u32(S.ring);
 #endif
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
-        const uint32_t ex = inc[j & 1] - packed[j & 1];
+        const int q = NPK * o + (j & 1);
+        const uint32_t ex = inc[q] - packed[q];
         int32_t p = rb + (int32_t)((ex >> (8 * (j >> 1))) & 0xFFu);
 #if RA_SEL_PTXSCATTER
         uint32_t a = ring0 + 4u * (uint32_t)p;  // byte address: one predicated store + add per row
@@ -572,24 +696,24 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
           // ROWS: the row id (n < 2^32 is checked by ra_select_rows)
           const int32_t val = ROWS ? (int32_t)(uint32_t)(t * SEL_TILE + warp * WROWS - P.mis + 4 * (32 * j + lane) + c)
                                    : comp(v[j], c);
-          put_if(a, fl, 1u << (4 * j + c), val);
+          put_if(a, f, 1u << (4 * j + c), val);
         }
 #else
-        const uint32_t bits = (fl >> (4 * j)) & 0xFu;
+        const uint32_t bits = (f >> (4 * j)) & 0xFu;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
           if (bits & (1u << c))
             S.ring[p++] = ROWS ? (int32_t)(uint32_t)(t * SEL_TILE + warp * WROWS - P.mis + 4 * (32 * j + lane) + c)
                                : comp(v[j], c);
 #endif
-        rb += (int32_t)((tot[j & 1] >> (8 * (j >> 1))) & 0xFFu);
+        rb += (int32_t)((tot[q] >> (8 * (j >> 1))) & 0xFFu);
       }
     }
-    wp = start + agg;
+    wp = start + rows_in;
     // ---- gather: tile i - LAG is due
     if (i - LAG >= head) {
-      write_tile<ROWS>(S, P, head, tid);
-      used -= S.cnt[head % K];
+      write_tile<ROWS, M, SM>(S, P, head, tid);
+      used -= S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0);
       ++head;
     }
   }
@@ -600,24 +724,24 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     mbar_arrive(&S.counted[i % K]);
   }
   compute_bar();  // scatters of the last tiles are visible
-  for (; head < i; ++head) write_tile<ROWS>(S, P, head, tid);
+  for (; head < i; ++head) write_tile<ROWS, M, SM>(S, P, head, tid);
 }
 
 struct KernelCfg {
-  int grid_per_sm[64][4];
+  int grid_per_sm[64][8];
 };
 KernelCfg g_cfg;
 
-template <bool HAS_NE, bool ROWS>
+template <bool HAS_NE, bool ROWS, int M>
 int ensure_config(int dev, int& per_sm) {
-  int& c = g_cfg.grid_per_sm[dev][(HAS_NE ? 1 : 0) + (ROWS ? 2 : 0)];
+  int& c = g_cfg.grid_per_sm[dev][(HAS_NE ? 1 : 0) + (ROWS ? 2 : 0) + (M == 2 ? 4 : 0)];
   if (!c) {
-    const int smem = (int)sizeof(SelSmem);
-    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE, ROWS>,
+    const int smem = (int)sizeof(SmemFor<M>);
+    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE, ROWS, M>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(select smem)");
     int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE, ROWS>, BLOCK, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE, ROWS, M>, BLOCK, smem);
     if (e != cudaSuccess) return cuda_fail(e, "occupancy(select)");
     if (occ < 1) return fail(RA_E_CUDA, "select kernel does not fit on an SM");
     c = occ;
@@ -643,15 +767,38 @@ int sel_ctas_per_sm() {
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) dev = 0;
   int per_sm = 0;
-  if (ensure_config<false, false>(dev, per_sm)) return -1;
+  if (ensure_config<false, false, 1>(dev, per_sm)) return -1;
   return per_sm;
 }
 
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, uint32_t* rows) {
+                       cudaStream_t s, uint32_t* rows, const SelSecond* second) {
   SelParams P;
   P.rowids = rows;
+  P.lo2 = 0;
+  P.span2 = 0;
+  P.n_ne2 = 0;
+  for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne2[j] = 0;
+  P.out2 = nullptr;
+  P.out_cap2 = 0;
+  P.d_count2 = nullptr;
+  if (second) {
+    const CanonPred& c2 = second->cp;
+    P.lo2 = c2.lo;
+    P.span2 = (uint32_t)c2.hi - (uint32_t)c2.lo;
+    P.n_ne2 = c2.n_ne;
+    for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne2[j] = j < c2.n_ne ? c2.ne[j] : 0;
+    if (c2.lo > c2.hi) {  // empty interval
+      P.lo2 = 0;
+      P.span2 = 0;
+      P.n_ne2 = 1;
+      P.ne2[0] = 0;
+    }
+    P.out2 = second->out;
+    P.out_cap2 = second->out_cap;
+    P.d_count2 = second->d_count;
+  }
   const uintptr_t a = (uintptr_t)d_in;
   P.mis = (int32_t)((a & 15u) >> 2);
   P.abase = (const int32_t*)(a - (a & 15u));
@@ -677,11 +824,23 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) dev = 0;
-  const bool ne = P.n_ne > 0;
+  const bool ne = P.n_ne > 0 || P.n_ne2 > 0;
   const bool rw = rows != nullptr;
+  const bool two = second != nullptr;
+  if (rw && two) return fail(RA_E_INVAL, "row-id mode has one output");
   int per_sm = 1;
-  int rc = rw ? (ne ? ensure_config<true, true>(dev, per_sm) : ensure_config<false, true>(dev, per_sm))
-              : (ne ? ensure_config<true, false>(dev, per_sm) : ensure_config<false, false>(dev, per_sm));
+  int rc;
+  const void* kern;
+  if (two) {
+    rc = ne ? ensure_config<true, false, 2>(dev, per_sm) : ensure_config<false, false, 2>(dev, per_sm);
+    kern = ne ? (const void*)select_fused_kernel<true, false, 2> : (const void*)select_fused_kernel<false, false, 2>;
+  } else if (rw) {
+    rc = ne ? ensure_config<true, true, 1>(dev, per_sm) : ensure_config<false, true, 1>(dev, per_sm);
+    kern = ne ? (const void*)select_fused_kernel<true, true, 1> : (const void*)select_fused_kernel<false, true, 1>;
+  } else {
+    rc = ne ? ensure_config<true, false, 1>(dev, per_sm) : ensure_config<false, false, 1>(dev, per_sm);
+    kern = ne ? (const void*)select_fused_kernel<true, false, 1> : (const void*)select_fused_kernel<false, false, 1>;
+  }
   if (rc) return rc;
   const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
   int64_t grid = (int64_t)num_sms() * per_sm;
@@ -689,12 +848,9 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   if (grid < 1) grid = 1;
   // Cooperative launch keeps the persistent CTAs co-resident (they wait on
   // each other's aggregates); tickets make the order independent of blockIdx.
-  const size_t smem = sizeof(SelSmem);
+  const size_t smem = two ? sizeof(SelSmem2) : sizeof(SelSmem);
   void* args[] = {(void*)&P};
-  cudaError_t le = cudaLaunchCooperativeKernel(
-      rw ? (ne ? (const void*)select_fused_kernel<true, true> : (const void*)select_fused_kernel<false, true>)
-         : (ne ? (const void*)select_fused_kernel<true, false> : (const void*)select_fused_kernel<false, false>),
-      dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
+  cudaError_t le = cudaLaunchCooperativeKernel(kern, dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
   if (le != cudaSuccess) return cuda_fail(le, "select_fused_kernel cooperative launch");
   count_launch();
   return RA_OK;

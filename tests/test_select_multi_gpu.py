@@ -1,0 +1,95 @@
+"""GPU parity of several SELECTs on one input (ra_select_multi, SURVEY §8(f)
+f2, Fig 2(c)) through the C-ABI against the CPU oracle (oracle.select_multi):
+each output bit-exact and in input order, over ragged/misaligned inputs, many
+tiles, every selectivity regime, != predicates, capacity limits, and
+interleaved with single-output calls on the same workspace."""
+import numpy as np
+import pytest
+
+import oracle
+import ragen
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def R():
+    import paper_conf_ipps_wudwcyc12_b200 as R
+    return R
+
+
+def check(R, x, chains, offset=0):
+    xd = torch.from_numpy(np.concatenate([np.zeros(offset, np.int32), x])).cuda()[offset:]
+    outs, cnt = R.select_multi(xd, chains)
+    torch.cuda.synchronize()
+    exp = oracle.select_multi(x, chains)
+    for o, (out, e) in enumerate(zip(outs, exp)):
+        c = int(cnt[o].item())
+        assert c == e.size, (o, c, e.size)
+        assert np.array_equal(out[:c].cpu().numpy(), e), o
+
+
+@pytest.mark.parametrize("n", [0, 1, 5, 8191, 8192, 8193, 5 * 8192 + 1234, 1_000_003])
+@pytest.mark.parametrize("offset", [0, 1, 2, 3])
+def test_sizes_offsets(R, n, offset):
+    x = ragen.int32_column(71 + n, n)
+    check(R, x, [[("lt", 0)], [("gt", -(2**29)), ("lt", 2**30)]], offset)
+
+
+@pytest.mark.parametrize("s0,s1", [(0.0, 1.0), (0.01, 0.9), (0.5, 0.5), (0.9, 0.9), (1.0, 1.0), (0.25, 0.75)])
+def test_selectivities_many_tiles(R, s0, s1):
+    n = (1 << 22) + 333
+    x = ragen.int32_column(72, n)
+
+    def chain(s):
+        if s == 0.0:
+            return [("lt", -(2**31))]
+        if s == 1.0:
+            return [("ge", -(2**31))]
+        return [("lt", ragen.nested_thresholds(s, 1)[0])]
+    check(R, x, [chain(s0), chain(s1)])
+
+
+def test_complementary_and_ne(R):
+    n = 2_000_001
+    x = ragen.int32_column(73, n)
+    t = int(x[999])
+    check(R, x, [[("lt", t)], [("ge", t)]])
+    check(R, x, [[("ne", int(x[5])), ("ne", int(x[6])), ("lt", 2**30)], [("eq", int(x[7]))]])
+    check(R, x, [[], [("le", 0)]])  # k = 0: identity output
+
+
+def test_single_output_and_shared_workspace(R):
+    n = 300_007
+    x = ragen.int32_column(74, n)
+    xd = torch.from_numpy(x).cuda()
+    check(R, x, [[("lt", 12345)]])
+    for _ in range(3):  # alternate single-output and dual-output launches on one workspace
+        out, c = R.select_chain(xd, [("gt", 0)])
+        outs, cnt = R.select_multi(xd, [[("lt", 0)], [("gt", 0)]])
+        torch.cuda.synchronize()
+        e = x[x > 0]
+        assert int(c.item()) == e.size and np.array_equal(out[:e.size].cpu().numpy(), e)
+        assert np.array_equal(outs[1][:int(cnt[1].item())].cpu().numpy(), e)
+
+
+def test_capacity(R):
+    n = 400_000
+    x = ragen.int32_column(75, n)
+    xd = torch.from_numpy(x).cuda()
+    outs = [torch.empty(1000, dtype=torch.int32, device="cuda"), torch.empty(n, dtype=torch.int32, device="cuda")]
+    outs, cnt = R.select_multi(xd, [[("lt", 0)], [("gt", 0)]], outs=outs)
+    torch.cuda.synchronize()
+    e0, e1 = x[x < 0], x[x > 0]
+    assert int(cnt[0].item()) == e0.size and int(cnt[1].item()) == e1.size
+    assert np.array_equal(outs[0].cpu().numpy(), e0[:1000])
+    assert np.array_equal(outs[1][:e1.size].cpu().numpy(), e1)
+
+
+def test_argument_errors(R):
+    xd = torch.zeros(16, dtype=torch.int32, device="cuda")
+    with pytest.raises(R.RAError) as e:
+        R.select_multi(xd, [[("lt", 0)]] * 3)
+    assert e.value.code == R.RA_E_INVAL

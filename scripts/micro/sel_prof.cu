@@ -5,6 +5,8 @@
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/capi.cu"
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/select_fused.cu"
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/q1_fused.cu"
+#include "../../paper_conf_ipps_wudwcyc12_b200/csrc/q1_narrow.cu"
+#include "../../paper_conf_ipps_wudwcyc12_b200/csrc/gather.cu"
 #include <cstdlib>
 #ifndef VARIANT
 #define VARIANT "full"

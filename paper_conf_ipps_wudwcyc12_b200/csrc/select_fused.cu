@@ -99,6 +99,9 @@ constexpr int BLOCK = SEL_THREADS + 64;  // + the look-back and producer warps
 #endif
 constexpr int LAG = RA_SEL_LAG;          // tile k is written when tile k+LAG is counted (or earlier)
 constexpr int K = LAG + 2;               // metadata slots: tiles counted but not yet written
+#ifndef RA_SEL_COOP
+#define RA_SEL_COOP 0
+#endif
 #ifndef RA_SEL_PTXSCATTER
 #define RA_SEL_PTXSCATTER 1
 #endif
@@ -846,12 +849,18 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   int64_t grid = (int64_t)num_sms() * per_sm;
   if (grid > ntiles_max) grid = ntiles_max;
   if (grid < 1) grid = 1;
-  // Cooperative launch keeps the persistent CTAs co-resident (they wait on
-  // each other's aggregates); tickets make the order independent of blockIdx.
+  // No co-residency is required (plain launch): a CTA only ever waits on the
+  // aggregates of tiles with lower tickets, tickets are drawn only by running
+  // CTAs, and a tile's aggregate is published before its CTA can block on
+  // any placement — so the lowest unpublished tile can always be published.
   const size_t smem = two ? sizeof(SelSmem2) : sizeof(SelSmem);
   void* args[] = {(void*)&P};
+#if RA_SEL_COOP
   cudaError_t le = cudaLaunchCooperativeKernel(kern, dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
-  if (le != cudaSuccess) return cuda_fail(le, "select_fused_kernel cooperative launch");
+#else
+  cudaError_t le = cudaLaunchKernel(kern, dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
+#endif
+  if (le != cudaSuccess) return cuda_fail(le, "select_fused_kernel launch");
   count_launch();
   return RA_OK;
 }

@@ -197,6 +197,16 @@ using dev::mbar_wait;
 using dev::mbar_test;
 using dev::bulk_g2s;
 
+__device__ __forceinline__ void st_relaxed_shared(int32_t* p, int32_t v) {
+  asm volatile("st.relaxed.cta.shared.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ int32_t ld_relaxed_shared(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.relaxed.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+
 // Compute warps synchronise among themselves only (named barrier 1).
 __device__ __forceinline__ void compute_bar() { asm volatile("bar.sync 1, %0;" ::"n"(SEL_THREADS) : "memory"); }
 
@@ -358,7 +368,9 @@ __device__ __forceinline__ void window_sum2(const SM& S, const SelParams& P, int
 // (ROWS mode: the run holds row ids).
 template <bool ROWS, int M, typename SM>
 __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int tid) {
-  if (tid == 0) *(volatile int*)&S.demand = k;  // tell the look-back warp not to wait for later counts
+  // tell the look-back warp not to wait for later counts (a monotone hint,
+  // relaxed accesses on both sides: never a plain racing access)
+  if (tid == 0) st_relaxed_shared(&S.demand, k);
   PT_BEGIN(t0);
   mbar_wait(&S.placed[k % K], (uint32_t)((k / K) & 1));
   PT_END(2, t0, tid == 0);
@@ -476,7 +488,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // tile k+D2 is counted — or at once when the compute warps already wait
     // for tile k (`demand`: ring of selected rows full at high selectivity).
     auto due = [&](int k, int d) {
-      return __all_sync(0xffffffffu, *(volatile int*)&S.demand >= k) || counted(k + d);
+      return __all_sync(0xffffffffu, ld_relaxed_shared(&S.demand) >= k) || counted(k + d);
     };
     int c_next = 0;  // next window to copy
     for (int k = 0;; ++k) {

@@ -60,6 +60,9 @@ __device__ __forceinline__ void warp_sum_u128(uint64_t& lo, uint64_t& hi) {
 // Reduction: warp (shuffles) -> CTA (smem) -> grid (last CTA, 128-bit fold).
 // Called by every thread of the CTA; warps >= NW (a producer warp) only join
 // the barriers.  s_w: [NW][NS][8] shared scratch.
+template <typename Params>
+__device__ __forceinline__ void publish_and_fold(const Params& P, bool* s_last);
+
 template <int NW, typename Params>
 __device__ __forceinline__ void reduce_and_fold(const Acc& A, const Params& P, uint64_t (*s_w)[NS][8],
                                                 uint32_t* s_status, bool* s_last) {
@@ -109,6 +112,13 @@ __device__ __forceinline__ void reduce_and_fold(const Acc& A, const Params& P, u
     }
   }
   if (threadIdx.x == 0) mine->status = *s_status;
+  publish_and_fold(P, s_last);
+}
+
+// After this CTA wrote its Q1Block: ticket; the last CTA to arrive folds all
+// CTA partials into *P.out (128-bit where needed).  Called by every thread.
+template <typename Params>
+__device__ __forceinline__ void publish_and_fold(const Params& P, bool* s_last) {
   __threadfence();
   __syncthreads();
   if (threadIdx.x == 0) *s_last = (atomicAdd(P.counter, 1u) == gridDim.x - 1);

@@ -44,7 +44,8 @@ using namespace q1c;
 constexpr int QN_NT = 256;     // compute threads + 1 producer warp
 constexpr int QN_NW = QN_NT / 32;
 constexpr int QN_TILE = 1024;  // rows per tile (11 KB)
-constexpr int QN_STAGES = 8;
+constexpr int QN_STAGES = 4;
+constexpr int QN_CTAS_PER_SM = 2;
 constexpr int QN_R = QN_TILE / QN_NT;  // 4 rows per thread per tile
 constexpr int QN_FLUSH_TILES = 256 / QN_R;
 static_assert(QN_R == 4, "the per-thread loads below take 4 rows");
@@ -74,18 +75,13 @@ struct QnParams {
 struct QnSmem {
   alignas(128) unsigned char stage[QN_STAGES][NSTAGE_BYTES];
   uint4 rec[NS + 1][2][QN_NT];  // [slot][half][thread]: thread-private 32-byte records
-  uint64_t s_w[QN_NW][NS][8];
+  unsigned long long wsum[NS][6];  // CTA sums: count, qty, price, disc, disc_price, charge
   uint64_t full[QN_STAGES], empty[QN_STAGES];
   uint32_t status;
   bool last;
 };
 constexpr size_t QN_SMEM = sizeof(QnSmem);
 static_assert(QN_SMEM <= 227 * 1024, "narrow Q1 kernel exceeds the shared-memory opt-in limit");
-
-struct NAcc {  // 64-bit per-thread totals (count and disc fit 32 bits: <= 2^17 rows/thread)
-  uint32_t cnt[NS], disc[NS];
-  uint64_t sq[NS], sp[NS], dp[NS], ch[NS];
-};
 
 __device__ __forceinline__ uint4 lds128(uint32_t a) {
   uint4 v;
@@ -126,28 +122,47 @@ __device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cu
   sts128(ra + REC_HALF, b);
 }
 
-// Fold the records into the 64-bit sums.  Between two flushes a thread adds
-// <= 256 rows, so every record field stays within 32 bits:
+// Fold the records into the CTA's 64-bit sums (warp REDUX + one shared atomic
+// per field per warp).  Between two
+// flushes a thread adds <= 256 rows, so every record field stays in 32 bits:
 //   count <= 256 (<< 16 -> < 2^25), disc <= 25600 < 2^16, qty < 2^16 * 2^8,
 //   price <= (2^24-1) * 2^8 < 2^32, dp>>16 < 2^15 * 2^8, dp&0xffff < 2^16 * 2^8,
 //   f*(dp>>16) < 200 * 2^15 * 2^8 < 2^31, f*(dp&0xffff) < 200 * 2^16 * 2^8 < 2^32.
-__device__ __forceinline__ void nflush(NAcc& W, uint32_t rec0) {
+// A CTA takes <= 2^24 rows (launch_q1_narrow), so its charge sum stays below
+// 200 * 100 * 2^24 * 2^24 < 2^63 and every CTA sum fits 64 bits.
+// Warp sum of 32-bit values as an exact 64-bit value: REDUX on the 16-bit
+// halves (each sum < 32 * 2^16, no overflow).
+__device__ __forceinline__ unsigned long long warp_sum32(uint32_t v) {
+  const uint32_t lo = __reduce_add_sync(0xffffffffu, v & 0xFFFFu);
+  const uint32_t hi = __reduce_add_sync(0xffffffffu, v >> 16);
+  return (unsigned long long)lo + ((unsigned long long)hi << 16);
+}
+
+__device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
+  const int lane = threadIdx.x & 31;
 #pragma unroll
   for (int s = 0; s < NS; ++s) {
     const uint32_t ra = rec0 + s * REC_SLOT;
     const uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
-    W.cnt[s] += a.x >> 16;
-    W.disc[s] += a.x & 0xFFFFu;
-    W.sq[s] += a.y;
-    W.sp[s] += a.z;
-    W.dp[s] += ((uint64_t)a.w << 16) + b.x;
-    W.ch[s] += ((uint64_t)b.y << 16) + b.z;
+    if (!__any_sync(0xffffffffu, (a.x | a.y | a.z | a.w | b.x | b.y | b.z) != 0u)) continue;  // warp-uniform
+    const unsigned long long cnt = warp_sum32(a.x >> 16), disc = warp_sum32(a.x & 0xFFFFu);
+    const unsigned long long q = warp_sum32(a.y), p = warp_sum32(a.z);
+    const unsigned long long dph = warp_sum32(a.w), dpl = warp_sum32(b.x);
+    const unsigned long long chh = warp_sum32(b.y), chl = warp_sum32(b.z);
+    if (lane == 0) {
+      atomicAdd(&S.wsum[s][0], cnt);
+      atomicAdd(&S.wsum[s][1], q);
+      atomicAdd(&S.wsum[s][2], p);
+      atomicAdd(&S.wsum[s][3], disc);
+      atomicAdd(&S.wsum[s][4], (dph << 16) + dpl);
+      atomicAdd(&S.wsum[s][5], (chh << 16) + chl);
+    }
     sts128(ra, make_uint4(0, 0, 0, 0));
     sts128(ra + REC_HALF, make_uint4(0, 0, 0, 0));
   }
 }
 
-__global__ void __launch_bounds__(QN_NT + 32, 1) q1n_kernel(const QnParams P) {
+__global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const QnParams P) {
   extern __shared__ __align__(128) unsigned char qn_smem_raw[];
   QnSmem& S = *reinterpret_cast<QnSmem*>(qn_smem_raw);
   const int tid = threadIdx.x;
@@ -164,10 +179,10 @@ __global__ void __launch_bounds__(QN_NT + 32, 1) q1n_kernel(const QnParams P) {
 #pragma unroll
     for (int s = 0; s <= NS; ++s) S.rec[s][0][tid] = S.rec[s][1][tid] = make_uint4(0, 0, 0, 0);
   }
+  if (tid < NS * 6) (&S.wsum[0][0])[tid] = 0ull;
+  if (tid == 0) S.status = 0;
   __syncthreads();
 
-  Acc A;
-  acc_zero(A);
   if (warp == QN_NW) {
     // ---------------- producer warp: one elected lane issues the bulk copies
     if (lane == 0) {
@@ -189,12 +204,6 @@ __global__ void __launch_bounds__(QN_NT + 32, 1) q1n_kernel(const QnParams P) {
     }
   } else {
     // ---------------- compute warps: rows 4*tid .. 4*tid+3 of each tile
-    NAcc N;
-#pragma unroll
-    for (int s = 0; s < NS; ++s) {
-      N.cnt[s] = N.disc[s] = 0;
-      N.sq[s] = N.sp[s] = N.dp[s] = N.ch[s] = 0;
-    }
     const uint32_t rec0 = dev::smem_u32(&S.rec[0][0][tid]);
     uint32_t status = 0;
     int i = 0, since = 0;
@@ -216,28 +225,39 @@ __global__ void __launch_bounds__(QN_NT + 32, 1) q1n_kernel(const QnParams P) {
            (t >> 16) & 0xFF, p.z);
       nrow(rec0, status, P.cutoff, sd.y >> 16, g >> 24, q.y >> 16, d >> 24, t >> 24, p.w);
       if (++since == QN_FLUSH_TILES) {
-        nflush(N, rec0);
+        nflush(S, rec0);
         since = 0;
       }
     }
-    nflush(N, rec0);
+    nflush(S, rec0);
     // tail rows after the full tiles (< 1 per thread)
     const int64_t tail0 = P.ntiles * QN_TILE;
     for (int64_t r = tail0 + (int64_t)blockIdx.x * QN_NT + tid; r < P.n; r += (int64_t)gridDim.x * QN_NT)
       nrow(rec0, status, P.cutoff, P.sd[r], P.g[r], P.q[r], P.d[r], P.t[r], P.p[r]);
-    nflush(N, rec0);
-#pragma unroll
-    for (int s = 0; s < NS; ++s) {
-      A.cnt[s] = N.cnt[s];
-      A.sdisc[s] = N.disc[s];
-      A.sq[s] = N.sq[s];
-      A.sp[s] = N.sp[s];
-      A.sdp[s] = N.dp[s];
-      A.sch[s] = N.ch[s];
-    }
-    A.status = status;
+    nflush(S, rec0);
+    if (status) atomicOr(&S.status, status);
   }
-  reduce_and_fold<QN_NW>(A, P, S.s_w, &S.status, &S.last);
+  // CTA partial -> P.blocks[blockIdx]; the last CTA folds all of them
+  __syncthreads();
+  if (tid < NS * 4) {
+    const int sl = tid >> 2, f = tid & 3;
+    Q1Block* mine = P.blocks + blockIdx.x;
+    if (f == 0) {
+      mine->v[sl][0] = S.wsum[sl][0];
+      mine->v[sl][1] = S.wsum[sl][1];
+    } else if (f == 1) {
+      mine->v[sl][2] = S.wsum[sl][2];
+      mine->v[sl][3] = S.wsum[sl][3];
+    } else if (f == 2) {
+      mine->v[sl][4] = S.wsum[sl][4];
+      mine->v[sl][5] = 0;
+    } else {
+      mine->v[sl][6] = S.wsum[sl][5];
+      mine->v[sl][7] = 0;
+    }
+  }
+  if (tid == 0) P.blocks[blockIdx.x].status = S.status;
+  publish_and_fold(P, &S.last);
 }
 
 // ------------------------------------------------------------- encoder
@@ -300,11 +320,11 @@ int launch_q1_narrow(const ra_lineitem_narrow& c, int64_t n, int32_t cutoff, ra_
     if (e != cudaSuccess) return cuda_fail(e, "q1n_kernel smem attribute");
     g_qn_attr[dev] = true;
   }
-  int64_t grid = num_sms();
+  int64_t grid = (int64_t)num_sms() * QN_CTAS_PER_SM;
   const int64_t need = P.ntiles > 0 ? P.ntiles : 1;
   if (grid > need) grid = need;
-  // per-thread sums stay exact while rows/thread <= 2^17
-  const int64_t min_grid = (n >> 17) / QN_NT + 1;
+  // CTA sums stay exact (< 2^63) while rows/CTA <= 2^24 (nflush)
+  const int64_t min_grid = (n >> 24) + 1;
   if (grid < min_grid) grid = min_grid;
   if (grid > Q1_MAX_GRID) return fail(RA_E_INVAL, "n too large for the Q1 grid");
   q1n_kernel<<<(unsigned)grid, QN_NT + 32, QN_SMEM, s>>>(P);

@@ -266,8 +266,8 @@ def run_ours(args, D: Dist):
 
 
 def extras(args, D, torch, R, x, preds, kept, chain_ms):
-    s_sel = args.sel
     """Other BASELINE configs + e2e + CPU baseline, same timing rules."""
+    s_sel = args.sel
     dev = x.device
     sh = int(torch.cuda.current_stream().cuda_stream)
     n = x.numel()

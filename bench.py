@@ -68,8 +68,17 @@ class Dist:
     def init(self, torch):
         if self.world > 1:
             import torch.distributed as dist
-            dist.init_process_group("nccl", device_id=torch.device("cuda", self.local))
+            # RA_BENCH_BACKEND=gloo: exercise the multi-rank code path with several
+            # ranks sharing one GPU (functional check only; NCCL needs one GPU per rank)
+            backend = os.environ.get("RA_BENCH_BACKEND", "nccl")
+            if backend == "nccl":
+                dist.init_process_group("nccl", device_id=torch.device("cuda", self.local))
+            else:
+                dist.init_process_group(backend)
             self.pg = dist
+
+    def device(self, torch) -> int:
+        return self.local % torch.cuda.device_count()
 
     def barrier(self, torch):
         if self.pg:
@@ -168,12 +177,16 @@ def ncu_traffic(key: str):
     return None
 
 
-def timed(torch, D: Dist, fn, steps: int, warmup: int, kernel_fn=None):
+def timed(torch, D: Dist, fn, steps: int, warmup: int, kernel_fn=None, join=None):
     """W warm-up steps; then EXACTLY `steps` steps between barrier+sync on both
     sides, CUDA events on the launching (current) stream; max over ranks.
-    Returns (ms_per_step, mean kernel ms or None)."""
+    `join()` (optional) makes the current stream wait for work a step left on
+    other streams, before the closing event.  Returns (ms_per_step, mean kernel
+    ms or None)."""
     for i in range(warmup):
         fn(i)
+    if join:
+        join()
     D.barrier(torch)
     s = torch.cuda.current_stream()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -188,6 +201,8 @@ def timed(torch, D: Dist, fn, steps: int, warmup: int, kernel_fn=None):
             fn(i, kernel_done=True)
         else:
             fn(i)
+    if join:
+        join()
     e1.record(s)
     e1.synchronize()
     D.barrier(torch)
@@ -203,10 +218,10 @@ def timed(torch, D: Dist, fn, steps: int, warmup: int, kernel_fn=None):
 def run_ours(args, D: Dist):
     import torch
     D.init(torch)
-    torch.cuda.set_device(D.local)
+    torch.cuda.set_device(D.device(torch))
     import paper_conf_ipps_wudwcyc12_b200 as R
 
-    dev = torch.device("cuda", D.local)
+    dev = torch.device("cuda", D.device(torch))
     stream = torch.cuda.current_stream()
     sh = int(stream.cuda_stream)
     n = 1 << args.rows_log2
@@ -219,27 +234,50 @@ def run_ours(args, D: Dist):
     x = torch.empty(n, dtype=torch.int32, device=dev)
     ragen.int32_column_dev(CHAIN_SEED, x, row0=D.rank * n, stream=sh)
     out = torch.empty(n, dtype=torch.int32, device=dev)
-    cnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    # step i's count lands in cnts[i & 1]: step i's exchange (side stream) reads
+    # it while step i+1's kernel runs; step i+2's kernel waits for that exchange
+    cnts = torch.zeros(2, dtype=torch.int64, device=dev)
     ws_bytes = R.ra_select_workspace_bytes(n, k, 1)
     ws = torch.zeros(ws_bytes, dtype=torch.uint8, device=dev)
     from paper_conf_ipps_wudwcyc12_b200 import dist as rdist
-    args_chain = (x.data_ptr(), n, P, k, 1, out.data_ptr(), n, cnt.data_ptr(), ws.data_ptr(), ws_bytes, sh)
+    args_chain = [(x.data_ptr(), n, P, k, 1, out.data_ptr(), n, cnts.data_ptr() + 8 * b, ws.data_ptr(), ws_bytes, sh)
+                  for b in range(2)]
+    side = torch.cuda.Stream(device=dev)
+    kdone = [torch.cuda.Event() for _ in range(2)]
+    xdone = [None, None]
+    gathered = [torch.zeros(D.world, dtype=torch.int64, device=dev) for _ in range(2)]
 
     def chain_kernel(i):
-        R.ra_select_chain(*args_chain)
+        R.ra_select_chain(*args_chain[i & 1])
 
     def chain_step(i, kernel_done=False):
         if not kernel_done:
             chain_kernel(i)
-        if D.pg:  # a9: gather per-rank counts -> exclusive scan -> global offsets
-            rdist.exchange_counts(cnt)
+        if D.pg:  # a9: gather per-rank counts -> exclusive scan -> global offsets,
+            b = i & 1  # overlapped with the next step's kernel
+            kdone[b].record(stream)
+            side.wait_event(kdone[b])
+            with torch.cuda.stream(side):
+                rdist.exchange_counts(cnts[b:b + 1], counts=gathered[b])
+                xdone[b] = torch.cuda.Event()
+                xdone[b].record(side)
+            if xdone[b ^ 1] is not None:  # the next kernel reuses the buffer step i-1's exchange read
+                stream.wait_event(xdone[b ^ 1])
+
+    def join():
+        if D.pg:
+            stream.wait_stream(side)
 
     torch.cuda.synchronize()
     launches0 = R.ra_kernel_launches()
-    with ClockSampler(D.local) as clk:
-        ms, kms = timed(torch, D, chain_step, args.steps, args.warmup, kernel_fn=chain_kernel)
+    with ClockSampler(D.device(torch)) as clk:
+        ms, kms = timed(torch, D, chain_step, args.steps, args.warmup, kernel_fn=chain_kernel, join=join)
     launches = R.ra_kernel_launches() - launches0 - args.warmup
+    last = (args.steps - 1) & 1
+    cnt = cnts[last:last + 1]
     kept = int(cnt.item())
+    if D.pg:
+        assert int(gathered[last][D.rank].item()) == kept
     value = D.world * n / (ms * 1e-3)
     peak, peak_src = peaks()
     alg_bytes = 4 * n + 4 * kept

@@ -36,13 +36,15 @@ def exclusive_offsets(counts) -> list[int]:
     return out
 
 
-def exchange_counts(count, group=None):
+def exchange_counts(count, group=None, counts=None):
     """all_gather one int64 count per rank; returns (counts tensor, this rank's
-    global offset, total) — the SELECT exchange (a9)."""
+    global offset, total) — the SELECT exchange (a9).  ``counts`` (int64[world],
+    optional) receives the gathered counts."""
     import torch
     import torch.distributed as dist
     world = dist.get_world_size(group)
-    counts = torch.zeros(world, dtype=torch.int64, device=count.device)
+    if counts is None:
+        counts = torch.empty(world, dtype=torch.int64, device=count.device)
     dist.all_gather_into_tensor(counts, count.reshape(1).to(torch.int64), group=group)
     offs = torch.cumsum(counts, 0) - counts
     rank = dist.get_rank(group)

@@ -105,11 +105,8 @@ constexpr int K = LAG + 2;               // metadata slots: tiles counted but no
 #ifndef RA_SEL_PTXSCATTER
 #define RA_SEL_PTXSCATTER 1
 #endif
-#ifndef RA_SEL_PRODSLEEP
-#define RA_SEL_PRODSLEEP 0
-#endif
-#ifndef RA_SEL_PREDRAW
-#define RA_SEL_PREDRAW 1
+#ifndef RA_SEL_BATCH
+#define RA_SEL_BATCH 1  // tiles per ticket (see the producer warp)
 #endif
 #ifndef RA_SEL_D1
 #define RA_SEL_D1 1
@@ -125,8 +122,11 @@ constexpr int LBW = 10;                  // window words per lane per pass
 constexpr int WIN_WORDS = RA_SEL_WIN;     // window slot capacity (status words)
 constexpr int PASS_WORDS = 32 * LBW;      // words summed per warp pass
 static_assert(WIN_WORDS % 2 == 0, "16-B granules");
-constexpr int NPK = SEL_VEC / 4;         // packed count words per lane (4 rows of 8 bits each)
-static_assert(SEL_VEC == 8, "per-j counts are packed as 2 words x 4 bytes; fl has 32 bits");
+constexpr int NPK = SEL_VEC / 4;         // packed count words per lane (4 bytes: one per vector j)
+static_assert(SEL_VEC == 8 || SEL_VEC == 4, "fl holds 4 bits per vector in 32 bits; counts in NPK words");
+// vector j's 8-bit count: word NPK*o + q_of(j), byte b_of(j) (see the packing below)
+__host__ __device__ constexpr int q_of(int j) { return NPK == 2 ? (j & 1) : 0; }
+__host__ __device__ constexpr int b_of(int j) { return NPK == 2 ? (j >> 1) : ((j >> 1) | ((j & 1) << 1)); }
 static_assert(NW <= 32, "one warp reduces the per-warp counts");
 static_assert(LAG >= D2 + 1, "a tile is placed before it is due");
 static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");  // (M == 2: 2 x SEL_TILE, SelSmem2)
@@ -437,32 +437,33 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // round trip overlaps the wait for that slot; a slot is refilled as soon as
     // the compute warps have read it (B1), giving up to SEL_INSLOTS tiles in flight.
     if (lane == 0) {
-#if RA_SEL_PREDRAW
-      int64_t tn = (int64_t)atomicAdd(P.ticket, 1ull);
-#endif
+      // Tickets come in batches of G consecutive tiles; the next batch is drawn
+      // as the current one starts, so an atomic's L2 round trip overlaps G
+      // tiles of work.  G = 1 (measured, 2^28 rows: G = 2 is 2-4% faster at
+      // overall selectivity <= .25 but 40% slower at .5/.9, where a drawn,
+      // not yet counted tile holds up every later tile's placement).
+      constexpr int G = RA_SEL_BATCH;
+      int64_t cur = (int64_t)atomicAdd(P.ticket, (unsigned long long)G);
+      int64_t nxt = 0;
+      int g = 0;
       for (int j = 0;; ++j) {
         const int s = j % SEL_INSLOTS;
         PT_BEGIN(t0);
-#if RA_SEL_PRODSLEEP
-        if (j >= SEL_INSLOTS) dev::mbar_wait_sleep(&S.empty[s], (uint32_t)((j / SEL_INSLOTS - 1) & 1), RA_SEL_PRODSLEEP);
-#else
         if (j >= SEL_INSLOTS) mbar_wait(&S.empty[s], (uint32_t)((j / SEL_INSLOTS - 1) & 1));
-#endif
         PT_END(11, t0, true);
-#if !RA_SEL_PREDRAW
-        const int64_t tn = (int64_t)atomicAdd(P.ticket, 1ull);
-#endif
+        if (g == G) {
+          cur = nxt;
+          g = 0;
+        }
+        const int64_t tn = cur + g;
         S.tile_of[s] = tn;
         if (tn >= ntiles) {  // end marker for the compute warps
           mbar_arrive(&S.full[s]);
           break;
         }
         issue_tile(S, P, nv, tn, s);
-#if RA_SEL_PREDRAW
-        PT_BEGIN(t1);
-        tn = (int64_t)atomicAdd(P.ticket, 1ull);
-        PT_END(12, t1, true);
-#endif
+        if (g == 0) nxt = (int64_t)atomicAdd(P.ticket, (unsigned long long)G);
+        ++g;
       }
     }
     return;
@@ -615,10 +616,14 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       const uint32_t f = o == 0 ? fl : fl2;
       uint32_t x = f - ((f >> 1) & 0x55555555u);
       x = (x & 0x33333333u) + ((x >> 2) & 0x33333333u);
-      packed[NPK * o] = x & 0x0F0F0F0Fu;
-      packed[NPK * o + 1] = (x >> 4) & 0x0F0F0F0Fu;
-      inc[NPK * o] = packed[NPK * o];
-      inc[NPK * o + 1] = packed[NPK * o + 1];
+      if (NPK == 2) {  // even j in word 0, odd j in word 1, byte j >> 1
+        packed[NPK * o] = x & 0x0F0F0F0Fu;
+        packed[NPK * o + 1] = (x >> 4) & 0x0F0F0F0Fu;
+      } else {  // 16 flag bits: bytes j0, j2, j1, j3
+        packed[NPK * o] = (x & 0x0F0Fu) | (((x >> 4) & 0x0F0Fu) << 16);
+      }
+#pragma unroll
+      for (int q = 0; q < NPK; ++q) inc[NPK * o + q] = packed[NPK * o + q];
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -701,9 +706,9 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
 #endif
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
-        const int q = NPK * o + (j & 1);
+        const int q = NPK * o + q_of(j);
         const uint32_t ex = inc[q] - packed[q];
-        int32_t p = rb + (int32_t)((ex >> (8 * (j >> 1))) & 0xFFu);
+        int32_t p = rb + (int32_t)((ex >> (8 * b_of(j))) & 0xFFu);
 #if RA_SEL_PTXSCATTER
         uint32_t a = ring0 + 4u * (uint32_t)p;  // byte address: one predicated store + add per row
 #pragma unroll
@@ -721,7 +726,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
             S.ring[p++] = ROWS ? (int32_t)(uint32_t)(t * SEL_TILE + warp * WROWS - P.mis + 4 * (32 * j + lane) + c)
                                : comp(v[j], c);
 #endif
-        rb += (int32_t)((tot[q] >> (8 * (j >> 1))) & 0xFFu);
+        rb += (int32_t)((tot[q] >> (8 * b_of(j))) & 0xFFu);
       }
     }
     wp = start + rows_in;

@@ -44,6 +44,21 @@ int main(int argc, char** argv) {
   printf("%-24s thr %-12d ms %.4f  GB/s %.0f  count %lld  ctas/sm %d smem %zu err=%s\n", VARIANT, p[k - 1].value, ms,
          (4.0 * n + 4.0 * c) / ms / 1e6, (long long)c, ra::sel_ctas_per_sm(), sizeof(ra::SelSmem),
          cudaGetErrorString(cudaGetLastError()));
+  {  // verify the last launch's output against a host filter (dev check)
+    int32_t* hx = (int32_t*)malloc(n * 4);
+    int32_t* ho = (int32_t*)malloc(n * 4);
+    cudaMemcpy(hx, x, n * 4, cudaMemcpyDeviceToHost);
+    cudaMemcpy(ho, out, c * 4, cudaMemcpyDeviceToHost);
+    int64_t m = 0, bad = 0;
+    for (int64_t i = 0; i < n; ++i) {
+      bool keep = true;
+      for (int j = 0; j < k; ++j) keep &= hx[i] < p[j].value;
+      if (keep) { if (m < c && ho[m] != hx[i]) ++bad; ++m; }
+    }
+    printf("  verify: expected count %lld, mismatches %lld -> %s\n", (long long)m, (long long)bad,
+           (m == c && bad == 0) ? "OK" : "FAIL");
+    free(hx); free(ho);
+  }
 #ifdef RA_SEL_PROFILE
   unsigned long long z[16];
   cudaMemcpyFromSymbol(z, ra::g_sel_prof, sizeof(z));

@@ -455,20 +455,23 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     PT = R.make_preds(preds)
     at = (x.data_ptr(), n, PT, k, 0, pl, 3, n, tc.data_ptr(), tws.data_ptr(), tws_b, sh)
     tms, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_rows(*at), 20, 3)
-    tkms = tms  # select + gather kernels back to back (the whole step)
+    tkms = tms  # select + gather/compaction kernels back to back (the whole step)
     tk = int(tc.item())
     assert tk == kept
-    # key read, ids written + read back, 3 fields gathered + written
-    talg = 4 * n + 2 * 4 * tk + 3 * 4 * tk + 3 * 4 * tk
+    dense = tk * 16 > n  # the device's choice (ra_select_rows, 4-byte fields)
+    if dense:  # key read, ids staged, order masks (n/8) written + read, 3 columns streamed, 3 fields written
+        talg = 4 * n + 4 * tk + 2 * (n // 8) + 3 * 4 * n + 3 * 4 * tk
+        kname = "select_fused_kernel<ROWS> + compact_kernel"
+    else:  # key read, ids written + read back, 3 fields gathered + written
+        talg = 4 * n + 2 * 4 * tk + 3 * 4 * tk + 3 * 4 * tk
+        kname = "select_fused_kernel<ROWS> + gather_kernel"
     tach = talg / (tkms * 1e-3) / 1e9
     ex["tuple_select"] = {"rows_per_s": D.world * n / (tms * 1e-3), "ms_per_step": tms, "kernel_ms": tkms,
-                          "fields": 3, "kept": tk,
-                          "roofline": {"kernel": "select_fused_kernel<ROWS> + gather_kernel", "bound": "hbm",
-                                       "achieved": tach,
+                          "fields": 3, "kept": tk, "payload_path": "compaction" if dense else "gather",
+                          "roofline": {"kernel": kname, "bound": "hbm", "achieved": tach,
                                        "peak": peak, "unit": "GB/s", "frac": tach / peak,
                                        "algorithmic_bytes_per_launch": talg,
-                                       "traffic": ncu_traffic(f"select_rows_k{k}_s{s_sel}_n{n.bit_length() - 1}"),
-                                       "note": "gathers read whole 32-B sectors: DRAM traffic > algorithmic bytes"}}
+                                       "traffic": ncu_traffic(f"select_rows_k{k}_s{s_sel}_n{n.bit_length() - 1}")}}
     del f1, f2, outs, tws
 
     # --- configs[0]: single SELECT on 2^20 rows, 50% (latency-bound, L2-resident)

@@ -225,8 +225,12 @@ int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const* h_chai
  * column store field 0 is the int32 key column and the other fields are
  * payload columns.  One fused pass evaluates the predicate chain on the key
  * and compacts the selected rows' ids (order-preserving, single pass with
- * decoupled look-back); a gather kernel on the same stream then writes each
- * payload field at those ids (the paper's stage 4 "gather", Fig 3).
+ * decoupled look-back), also leaving per-tile order masks in the workspace;
+ * the payload fields are then placed on the same stream (the paper's stage 4
+ * "gather", Fig 3) by one of two kernels, chosen on the device from
+ * the count: few selected rows -> a gather at the ids; many -> a streaming
+ * compaction that reads each payload column once, in order.  Both give the
+ * same result (environment RA_TUPLE_GATHER=1 forces the gather: diagnostics).
  * With k = 0 every row is kept: PROJECT (Table I) of the payload
  * fields.  Output = the selected tuples, stream-ordered.
  *

@@ -4,6 +4,7 @@
 
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "ra_internal.cuh"
@@ -208,8 +209,10 @@ RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const*
 
 RA_API size_t ra_select_rows_workspace_bytes(int64_t n, int k) {
   if (n < 0) n = 0;
-  // select status words, then a staging area for the row ids
-  return ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256 + (((size_t)n * 4 + 255) / 256) * 256;
+  // select status words, then the per-tile masks for the payload compaction
+  // (and, for the A/B against the id gather, a staging area for the row ids)
+  return ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256 + ((ra::sel_masks_bytes(n) + 255) / 256) * 256 +
+         (((size_t)n * 4 + 255) / 256) * 256;
 }
 
 RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_preds, int k, uint32_t* d_rowids,
@@ -231,6 +234,8 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
   GatherSpec g;
   g.m = m;
+  g.n = n;
+  g.sparse_den = 16;  // 4-byte fields: gather below 1/16 selected (measured crossover)
   for (int j = 0; j < m; ++j) {
     const ra_payload& p = h_payloads[j];
     if (p.elem_bytes != 4 && p.elem_bytes != 8)
@@ -241,18 +246,32 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
     g.elem_bytes[j] = p.elem_bytes;
     g.col[j] = p.col;
     g.out[j] = p.out;
+    if (p.elem_bytes == 8) g.sparse_den = 3;  // 8-byte fields: sectors hold 4 rows, gather pays longer
   }
   CanonPred cp;
   rc = canonicalize(h_preds, k, &cp);
   if (rc) return rc;
-  // ids go to the caller's buffer, or (payload only) to the workspace staging area
-  const size_t stage_off = ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256;
+  if (getenv("RA_TUPLE_GATHER")) g.sparse_den = 0;  // A/B only: always the id gather
+  // One fused pass over the key writes the row ids (the caller's, or staged
+  // when only payloads are asked for) and the per-tile order masks; then the
+  // payload fields are placed by the gather or by the streaming compaction,
+  // chosen on the device from the count.
+  const size_t mask_off = ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256;
+  const size_t stage_off = mask_off + ((ra::sel_masks_bytes(n) + 255) / 256) * 256;
   uint32_t* ids = d_rowids ? d_rowids : (uint32_t*)((char*)d_ws + stage_off);
   const int64_t cap = d_rowids ? out_cap : (out_cap < n ? out_cap : n);
+  const int64_t T = ra::sel_max_tiles(n);
+  char* mb = (char*)d_ws + mask_off;
+  ra::SelMasks mk;
+  mk.fmask = (uint32_t*)mb;
+  mk.meta = (uint32_t*)(mb + (((size_t)T * SEL_THREADS * 4 + 255) / 256) * 256);
   rc = launch_select_pass(d_key, n, nullptr, cp, nullptr, cap, d_count, d_ws, (cudaStream_t)stream,
-                          (cap > 0 || !d_rowids) ? ids : nullptr);
+                          (cap > 0 || !d_rowids) ? ids : nullptr, nullptr,
+                          m > 0 && g.sparse_den > 0 ? &mk : nullptr);
   if (rc) return rc;
-  return launch_gather(ids, d_count, out_cap < n ? out_cap : n, g, (cudaStream_t)stream);
+  rc = launch_gather(ids, d_count, out_cap < n ? out_cap : n, g, (cudaStream_t)stream);
+  if (rc || g.sparse_den == 0) return rc;
+  return ra::launch_compact(d_key, n, mk, d_count, out_cap, g, (cudaStream_t)stream);
 }
 
 RA_API size_t ra_q1_workspace_bytes(int64_t n) {

@@ -24,6 +24,7 @@ __global__ void __launch_bounds__(GATHER_T) gather_kernel(const uint32_t* __rest
                                                           const int64_t* __restrict__ d_count, int64_t cap,
                                                           const GatherSpec g) {
   int64_t cnt = *d_count;
+  if (cnt * g.sparse_den > g.n) return;  // dense: compact_kernel places the fields
   if (cnt > cap) cnt = cap;
   const int64_t step = (int64_t)gridDim.x * GATHER_T * GATHER_U;
   for (int64_t base = (int64_t)blockIdx.x * GATHER_T * GATHER_U; base < cnt; base += step) {

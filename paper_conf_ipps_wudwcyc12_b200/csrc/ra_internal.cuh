@@ -70,19 +70,40 @@ struct SelSecond {
   int64_t out_cap;
   int64_t* d_count;
 };
+// Row-id mode extras for the payload compaction (compact.cu), per select tile t
+// (SEL_TILE rows counted from the key's 16-B aligned base): the compute lanes'
+// flag words fmask[t*SEL_THREADS + tid] and a 48-B record meta[t*12 ..]: the
+// compute warps' exclusive bases within the tile (u32 [0..8)) and the tile's
+// output offset (int64 at u32 index 8).
+struct SelMasks {
+  uint32_t* fmask;
+  uint32_t* meta;
+};
+size_t sel_masks_bytes(int64_t n);
+
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, uint32_t* rows = nullptr, const SelSecond* second = nullptr);
+                       cudaStream_t s, uint32_t* rows = nullptr, const SelSecond* second = nullptr,
+                       const SelMasks* masks = nullptr);
 
-// Gather of payload fields at row ids (the gather stage of a tuple SELECT):
-// out_j[i] = col_j[ids[i]] for i < min(*d_count, cap).
+// Payload fields of a tuple SELECT.  The selectivity decides, on the device,
+// which of the two kernels launched back to back places them: the id gather
+// when count * sparse_den <= n (few rows: read only their sectors), else the
+// streaming compaction (read each column once, in order).
 struct GatherSpec {
   int m;
   int32_t elem_bytes[RA_MAX_PAYLOAD];
   const void* col[RA_MAX_PAYLOAD];
   void* out[RA_MAX_PAYLOAD];
+  int64_t n;           // rows of the relation
+  int32_t sparse_den;  // see above (0: the gather always runs)
 };
+// Gather of payload fields at row ids (the gather stage of a tuple SELECT):
+// out_j[i] = col_j[ids[i]] for i < min(*d_count, cap).
 int launch_gather(const uint32_t* ids, const int64_t* d_count, int64_t cap, const GatherSpec& g, cudaStream_t s);
+// Payload compaction from the select pass's SelMasks (compact.cu).
+int launch_compact(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count, int64_t cap,
+                   const GatherSpec& g, cudaStream_t s);
 
 // Fused or unfused chain (validated arguments); used by the C-ABI and fission.
 int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,

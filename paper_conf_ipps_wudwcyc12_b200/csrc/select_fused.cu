@@ -142,7 +142,11 @@ struct SelParams {
   unsigned long long* ticket;
   uint64_t* status;  // status[tile]
   int32_t mis;       // rows of d_in's 16-B chunk before d_in (0..3)
-  uint32_t* rowids;  // ROWS mode (ra_select_rows): the ring holds row ids, written here
+  uint32_t* rowids;  // ROWS mode (ra_select_rows): the ring holds row ids, written here (or NULL)
+  // ROWS mode, payload compaction (compact.cu): per tile the lanes' flag words
+  // fmask[t][256] and meta[t][12] = the warps' exclusive bases + the tile offset
+  uint32_t* fmask;
+  uint32_t* meta;
   // M == 2 (ra_select_multi): a second predicate and output on the same input
   int32_t lo2;
   uint32_t span2;
@@ -376,6 +380,8 @@ __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int
   PT_END(2, t0, tid == 0);
   const int64_t g = S.goff[k % K];
   const int32_t c = S.cnt[k % K];
+  if (ROWS && P.meta && tid == 0) *reinterpret_cast<int64_t*>(P.meta + S.tidx[k % K] * 12 + 8) = g;
+  if (ROWS && !P.rowids) return;  // ids not requested: nothing in the ring
   const int32_t* run = S.ring + S.start[k % K];  // contiguous, never wraps
   int64_t lim = P.out_cap - g;
   lim = lim < 0 ? 0 : (lim > c ? c : lim);
@@ -605,6 +611,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         }
       }
     }
+    if (ROWS && P.fmask) P.fmask[t * SEL_THREADS + tid] = fl;  // for the payload compaction
     // ---- buffer: order (warp, j, lane, c); packed per-j counts, warp scans.
     // SWAR popcount of each nibble of fl (nibble j = the lane's 4 rows of
     // vector j), then j goes to word j&1, byte j>>1 (8 bits: a warp total <= 128).
@@ -658,7 +665,9 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       agg2 = (int32_t)__reduce_add_sync(0xffffffffu, wt2);
       wbase2 = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt2 : 0u);
     }
-    const int32_t rows_in = agg + agg2;  // ring rows this tile needs (both runs)
+    if (ROWS && P.meta && lane == 0) P.meta[t * 12 + warp] = (uint32_t)wbase;
+    const bool ring_rows = !ROWS || P.rowids;  // ROWS without ids: placement only, no ring
+    const int32_t rows_in = ring_rows ? agg + agg2 : 0;  // ring rows this tile needs (both runs)
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
       mbar_arrive(&S.empty[slot]);  // input slot free: the producer refills it
       const uint64_t aggw = M == 2 ? ((uint64_t)agg | ((uint64_t)agg2 << 16)) : (uint64_t)agg;
@@ -689,7 +698,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         break;
       }
       write_tile<ROWS, M, SM>(S, P, head, tid);
-      used -= S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0);
+      used -= ring_rows ? S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0) : 0;
       ++head;
       forced = true;
     }
@@ -698,7 +707,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     used += rows_in;
     // ---- scatter the tile into the ring (M == 2: the second run after the first)
 #pragma unroll
-    for (int o = 0; o < M; ++o) {
+    for (int o = 0; o < (ring_rows ? M : 0); ++o) {
       const uint32_t f = o == 0 ? fl : fl2;
       int32_t rb = start + (o == 0 ? wbase : agg + wbase2);
 #if RA_SEL_PTXSCATTER
@@ -733,7 +742,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ---- gather: tile i - LAG is due
     if (i - LAG >= head) {
       write_tile<ROWS, M, SM>(S, P, head, tid);
-      used -= S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0);
+      used -= ring_rows ? S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0) : 0;
       ++head;
     }
   }
@@ -793,9 +802,11 @@ int sel_ctas_per_sm() {
 
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, uint32_t* rows, const SelSecond* second) {
+                       cudaStream_t s, uint32_t* rows, const SelSecond* second, const SelMasks* masks) {
   SelParams P;
   P.rowids = rows;
+  P.fmask = masks ? masks->fmask : nullptr;
+  P.meta = masks ? masks->meta : nullptr;
   P.lo2 = 0;
   P.span2 = 0;
   P.n_ne2 = 0;
@@ -845,7 +856,7 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) dev = 0;
   const bool ne = P.n_ne > 0 || P.n_ne2 > 0;
-  const bool rw = rows != nullptr;
+  const bool rw = rows != nullptr || masks != nullptr;
   const bool two = second != nullptr;
   if (rw && two) return fail(RA_E_INVAL, "row-id mode has one output");
   int per_sm = 1;

@@ -94,6 +94,70 @@ def test_capacity_truncates_but_counts(R):
     assert np.array_equal(outs[0][:cap].cpu().numpy(), key[exp_ids[:cap]])
 
 
+@pytest.mark.parametrize("koff,poff", [(0, 0), (1, 1), (3, 3), (2, 0), (0, 3), (1, 2)])
+def test_payload_alignment_phases(R, koff, poff):
+    """Payload columns whose 16-B phase equals the key's take 128-bit loads,
+    the others element loads; both place every field exactly."""
+    n = 24 * 8192 + 1001
+    key = ragen.int32_column(66, n)
+    p4 = ragen.int32_column(67, n)
+    p8 = p4.astype(np.int64) * 7 + 1
+
+    def dev(a, off):
+        return torch.from_numpy(np.concatenate([np.zeros(off, a.dtype), a])).cuda()[off:]
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 2)]
+    ids, outs, cnt = R.select_rows(dev(key, koff), preds, [dev(p4, poff), dev(p8, poff), dev(key, poff)])
+    torch.cuda.synchronize()
+    c = int(cnt.item())
+    exp_ids, exp = oracle.select_rows(key, preds, [p4, p8, key])
+    assert c == exp_ids.size
+    assert np.array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
+    for o, e in zip(outs, exp):
+        assert np.array_equal(o[:c].cpu().numpy(), e)
+
+
+@pytest.mark.parametrize("cap", [1, 777, 8192 * 3 + 5])
+def test_capacity_never_writes_past_cap(R, cap):
+    n = 300_000
+    key = ragen.int32_column(68, n)
+    pay = (np.arange(n, dtype=np.int64) << 20) + 3
+    kd, pd = torch.from_numpy(key).cuda(), torch.from_numpy(pay).cuda()
+    preds = [("gt", -(2**30))]
+    exp_ids, (exp,) = oracle.select_rows(key, preds, [pay])
+    ids = torch.full((cap + 64,), 0xABCDEF, dtype=torch.int32, device="cuda")
+    out = torch.full((cap + 64,), -9, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    pl = (R.ra_payload * 1)()
+    pl[0].col, pl[0].out, pl[0].elem_bytes = pd.data_ptr(), out.data_ptr(), 8
+    wsb = R.ra_select_rows_workspace_bytes(n, 1)
+    ws = torch.zeros(wsb, dtype=torch.uint8, device="cuda")
+    R.ra_select_rows(kd.data_ptr(), n, R.make_preds(preds), 1, ids.data_ptr(), pl, 1, cap, cnt.data_ptr(),
+                     ws.data_ptr(), wsb, 0)
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == exp_ids.size
+    assert np.array_equal(ids[:cap].cpu().numpy().astype(np.int64), exp_ids[:cap])
+    assert np.array_equal(out[:cap].cpu().numpy(), exp[:cap])
+    assert (ids[cap:].cpu().numpy() == 0xABCDEF).all() and (out[cap:].cpu().numpy() == -9).all()
+
+
+@pytest.mark.parametrize("s", [0.03, 0.25, 0.6])
+@pytest.mark.parametrize("force_gather", [False, True])
+def test_both_payload_paths(R, s, force_gather, monkeypatch):
+    """The device picks the id gather (sparse) or the streaming compaction
+    (dense) from the count; RA_TUPLE_GATHER forces the gather.  Both are exact
+    for 4- and 8-byte fields, at selectivities on either side of the switch."""
+    if force_gather:
+        monkeypatch.setenv("RA_TUPLE_GATHER", "1")
+    else:
+        monkeypatch.delenv("RA_TUPLE_GATHER", raising=False)
+    n = 40 * 8192 + 4321
+    key = ragen.int32_column(69, n)
+    p4 = ragen.int32_column(70, n)
+    preds = [("lt", t) for t in ragen.nested_thresholds(s, 1)]
+    check(R, key, preds, [p4, key])  # 4-byte fields only
+    check(R, key, preds, [p4.astype(np.int64) * 5 - 7, p4])  # with an 8-byte field
+
+
 def test_argument_errors(R):
     kd = torch.zeros(16, dtype=torch.int32, device="cuda")
     bad = torch.zeros(16, dtype=torch.int16, device="cuda")

@@ -458,9 +458,9 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     tkms = tms  # select + gather/compaction kernels back to back (the whole step)
     tk = int(tc.item())
     assert tk == kept
-    dense = tk * 16 > n  # the device's choice (ra_select_rows, 4-byte fields)
-    if dense:  # key read, ids staged, order masks (n/8) written + read, 3 columns streamed, 3 fields written
-        talg = 4 * n + 4 * tk + 2 * (n // 8) + 3 * 4 * n + 3 * 4 * tk
+    dense = tk * 32 > n  # the device's choice (ra_select_rows, 4-byte fields)
+    if dense:  # key read, order masks (n/8) written + read, 3 columns streamed, 3 fields written
+        talg = 4 * n + 2 * (n // 8) + 3 * 4 * n + 3 * 4 * tk
         kname = "select_fused_kernel<ROWS> + compact_kernel"
     else:  # key read, ids written + read back, 3 fields gathered + written
         talg = 4 * n + 2 * 4 * tk + 3 * 4 * tk + 3 * 4 * tk

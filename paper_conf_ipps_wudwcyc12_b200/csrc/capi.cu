@@ -235,7 +235,7 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   GatherSpec g;
   g.m = m;
   g.n = n;
-  g.sparse_den = 16;  // 4-byte fields: gather below 1/16 selected (measured crossover)
+  g.sparse_den = 32;  // 4-byte fields: gather below 1/32 selected (measured crossover)
   for (int j = 0; j < m; ++j) {
     const ra_payload& p = h_payloads[j];
     if (p.elem_bytes != 4 && p.elem_bytes != 8)
@@ -246,16 +246,17 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
     g.elem_bytes[j] = p.elem_bytes;
     g.col[j] = p.col;
     g.out[j] = p.out;
-    if (p.elem_bytes == 8) g.sparse_den = 3;  // 8-byte fields: sectors hold 4 rows, gather pays longer
+    if (p.elem_bytes == 8) g.sparse_den = 8;  // 8-byte fields: sectors hold 4 rows, gather pays longer
   }
   CanonPred cp;
   rc = canonicalize(h_preds, k, &cp);
   if (rc) return rc;
   if (getenv("RA_TUPLE_GATHER")) g.sparse_den = 0;  // A/B only: always the id gather
-  // One fused pass over the key writes the row ids (the caller's, or staged
-  // when only payloads are asked for) and the per-tile order masks; then the
-  // payload fields are placed by the gather or by the streaming compaction,
-  // chosen on the device from the count.
+  // One fused pass over the key writes the caller's row ids (if asked for) and
+  // the per-tile order masks; then the payload fields are placed by the gather
+  // (sparse; ids rebuilt from the masks into the workspace when the caller
+  // did not ask for them) or by the streaming compaction (dense), chosen on
+  // the device from the count.
   const size_t mask_off = ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256;
   const size_t stage_off = mask_off + ((ra::sel_masks_bytes(n) + 255) / 256) * 256;
   uint32_t* ids = d_rowids ? d_rowids : (uint32_t*)((char*)d_ws + stage_off);
@@ -265,10 +266,15 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   ra::SelMasks mk;
   mk.fmask = (uint32_t*)mb;
   mk.meta = (uint32_t*)(mb + (((size_t)T * SEL_THREADS * 4 + 255) / 256) * 256);
+  const bool masks = m > 0 && g.sparse_den > 0;
+  const bool stage = !d_rowids && !masks;  // A/B: ids staged by the key pass
   rc = launch_select_pass(d_key, n, nullptr, cp, nullptr, cap, d_count, d_ws, (cudaStream_t)stream,
-                          (cap > 0 || !d_rowids) ? ids : nullptr, nullptr,
-                          m > 0 && g.sparse_den > 0 ? &mk : nullptr);
+                          (d_rowids && cap > 0) || stage ? ids : nullptr, nullptr, masks ? &mk : nullptr);
   if (rc) return rc;
+  if (masks && !d_rowids) {
+    rc = ra::launch_ids_from_masks(d_key, n, mk, d_count, g.sparse_den, ids, (cudaStream_t)stream);
+    if (rc) return rc;
+  }
   rc = launch_gather(ids, d_count, out_cap < n ? out_cap : n, g, (cudaStream_t)stream);
   if (rc || g.sparse_den == 0) return rc;
   return ra::launch_compact(d_key, n, mk, d_count, out_cap, g, (cudaStream_t)stream);

@@ -83,6 +83,28 @@ __device__ __forceinline__ void put_if_global(unsigned long long*& a, uint32_t f
       : "memory");
 }
 
+// The lane's exclusive (ex) and the warp's total (tot) packed counts of its
+// flag word (as select_fused.cu): vector j's count at word j & 1, byte j >> 1.
+__device__ __forceinline__ void packed_scan(uint32_t fl, int lane, uint32_t (&ex)[2], uint32_t (&tot)[2]) {
+  uint32_t x = fl - ((fl >> 1) & 0x55555555u);  // nibble popcounts
+  x = (x & 0x33333333u) + ((x >> 2) & 0x33333333u);
+  const uint32_t pk[2] = {x & 0x0F0F0F0Fu, (x >> 4) & 0x0F0F0F0Fu};  // even j | odd j
+  uint32_t inc[2] = {pk[0], pk[1]};
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc[q], d);
+      if (lane >= d) inc[q] += y;
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < 2; ++q) {
+    ex[q] = inc[q] - pk[q];
+    tot[q] = __shfl_sync(0xffffffffu, inc[q], 31);
+  }
+}
+
 // Place the flagged elements of the lane's SEL_VEC vectors (rows of vector j:
 // virtual vbase + 4*(32j + lane) + c) at out[dst0 + slice-local position].
 template <typename T>
@@ -200,20 +222,8 @@ __global__ void __launch_bounds__(CT_BLOCK, 2) compact_kernel(const CompactParam
       const bool mine = P.eb[f] == 4 || (warp >> 2) == h;
       if (mine && __any_sync(0xffffffffu, fl != 0u) && dst0 < cnt) {
         const int32_t lim = cnt - dst0 < SLICE ? (int32_t)(cnt - dst0) : SLICE;
-        uint32_t x = fl - ((fl >> 1) & 0x55555555u);  // packed per-vector counts (select_fused.cu)
-        x = (x & 0x33333333u) + ((x >> 2) & 0x33333333u);
-        const uint32_t pk[2] = {x & 0x0F0F0F0Fu, (x >> 4) & 0x0F0F0F0Fu};  // even j | odd j, byte j >> 1
-        uint32_t inc[2] = {pk[0], pk[1]};
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-#pragma unroll
-          for (int q = 0; q < 2; ++q) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc[q], d);
-            if (lane >= d) inc[q] += y;
-          }
-        }
-        const uint32_t ex[2] = {inc[0] - pk[0], inc[1] - pk[1]};
-        const uint32_t tot[2] = {__shfl_sync(0xffffffffu, inc[0], 31), __shfl_sync(0xffffffffu, inc[1], 31)};
+        uint32_t ex[2], tot[2];
+        packed_scan(fl, lane, ex, tot);
         // the warp's slice in the staged unit
         const int4* tile = !P.vec[f] ? nullptr
                            : P.eb[f] == 4 ? &S.data[s][warp * (SLICE / 4)] : &S.data[s][(warp & 3) * (SLICE / 2)];
@@ -228,7 +238,65 @@ __global__ void __launch_bounds__(CT_BLOCK, 2) compact_kernel(const CompactParam
   }
 }
 
+// Sparse path, no ids from the key pass: ids[i] = row of the i-th selected
+// tuple, from the order masks (one warp per 1024-row slice; predicated stores).
+__global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ fmask, const uint32_t* __restrict__ meta,
+                                                  const int64_t* __restrict__ d_count, int64_t n, int32_t mis,
+                                                  int32_t sparse_den, uint32_t* __restrict__ ids) {
+  const int64_t cnt = *d_count;
+  if (cnt * sparse_den > n) return;  // dense: compact_kernel places the fields, no ids needed
+  const int lane = threadIdx.x & 31;
+  const int64_t nslices = (n + mis + SLICE - 1) / SLICE;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
+  const int64_t w0 = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+  constexpr int U = 4;  // slices per warp iteration: their loads are issued together
+  for (int64_t sb = w0 * U; sb < nslices; sb += nw * U) {
+    uint32_t fl[U];
+    int64_t dst0[U];
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      const int64_t sl = sb + q;
+      fl[q] = sl < nslices ? __ldg(fmask + sl * 32 + lane) : 0u;
+      const int64_t t = sl / CT_WARPS;
+      dst0[q] = sl < nslices ? __ldg(reinterpret_cast<const long long*>(meta + t * 12 + 8)) +
+                                   __ldg(meta + t * 12 + sl % CT_WARPS)
+                             : 0;
+    }
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      if (!__any_sync(0xffffffffu, fl[q] != 0u)) continue;
+      uint32_t ex[2], tot[2];
+      packed_scan(fl[q], lane, ex, tot);
+      const uint32_t r0 = (uint32_t)((sb + q) * SLICE - mis);  // row of the slice's first virtual row (mod 2^32)
+      uint32_t* a0 = ids + dst0[q];
+      int32_t rb = 0;
+#pragma unroll
+      for (int j = 0; j < SEL_VEC; ++j) {  // sparse: visit the set bits only
+        uint32_t* a = a0 + rb + ((ex[j & 1] >> (8 * (j >> 1))) & 0xFFu);
+        for (uint32_t nib = (fl[q] >> (4 * j)) & 0xFu; nib; nib &= nib - 1u)
+          *a++ = r0 + 4 * (32 * j + lane) + (__ffs(nib) - 1);
+        rb += (int32_t)((tot[j & 1] >> (8 * (j >> 1))) & 0xFFu);
+      }
+    }
+  }
+}
+
 }  // namespace
+
+int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count,
+                          int32_t sparse_den, uint32_t* ids, cudaStream_t s) {
+  if (n == 0) return RA_OK;
+  const int32_t mis = (int32_t)(((uintptr_t)d_key & 15u) >> 2);
+  const int64_t nslices = (n + mis + SLICE - 1) / SLICE;
+  int64_t grid = (nslices + 31) / 32;  // 8 warps x 4 slices per CTA iteration
+  const int64_t lim = (int64_t)num_sms() * 8;
+  if (grid > lim) grid = lim;
+  ids_kernel<<<(unsigned)grid, 256, 0, s>>>(mk.fmask, mk.meta, d_count, n, mis, sparse_den, ids);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "ids_kernel launch");
+  return RA_OK;
+}
 
 size_t sel_masks_bytes(int64_t n) {
   const int64_t T = sel_max_tiles(n);

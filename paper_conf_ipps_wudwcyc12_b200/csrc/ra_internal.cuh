@@ -101,6 +101,10 @@ struct GatherSpec {
 // Gather of payload fields at row ids (the gather stage of a tuple SELECT):
 // out_j[i] = col_j[ids[i]] for i < min(*d_count, cap).
 int launch_gather(const uint32_t* ids, const int64_t* d_count, int64_t cap, const GatherSpec& g, cudaStream_t s);
+// Sparse path without caller ids: the row ids from the select pass's SelMasks
+// (exits on the device when the count is dense).
+int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count,
+                          int32_t sparse_den, uint32_t* ids, cudaStream_t s);
 // Payload compaction from the select pass's SelMasks (compact.cu).
 int launch_compact(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count, int64_t cap,
                    const GatherSpec& g, cudaStream_t s);

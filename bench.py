@@ -177,6 +177,15 @@ def ncu_traffic(key: str):
     return None
 
 
+def tuple_traffic(dense: bool, k, s_sel, lg):
+    """dram bytes of the tuple SELECT step: key pass + (compaction), from ncu."""
+    a = ncu_traffic(f"select_rows_k{k}_s{s_sel}_n{lg}")
+    if not dense or a is None:
+        return a
+    b = ncu_traffic(f"compact_k{k}_s{s_sel}_n{lg}")
+    return None if b is None else a + b
+
+
 def timed(torch, D: Dist, fn, steps: int, warmup: int, kernel_fn=None, join=None):
     """W warm-up steps; then EXACTLY `steps` steps between barrier+sync on both
     sides, CUDA events on the launching (current) stream; max over ranks.
@@ -471,7 +480,7 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                           "roofline": {"kernel": kname, "bound": "hbm", "achieved": tach,
                                        "peak": peak, "unit": "GB/s", "frac": tach / peak,
                                        "algorithmic_bytes_per_launch": talg,
-                                       "traffic": ncu_traffic(f"select_rows_k{k}_s{s_sel}_n{n.bit_length() - 1}")}}
+                                       "traffic": tuple_traffic(dense, k, s_sel, n.bit_length() - 1)}}
     del f1, f2, outs, tws
 
     # --- configs[0]: single SELECT on 2^20 rows, 50% (latency-bound, L2-resident)

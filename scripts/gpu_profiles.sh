@@ -8,3 +8,4 @@ $NCU --set full --import-source on --clock-control none -k regex:select_fused -s
 $NCU --set full --import-source on --clock-control none -k regex:q1_tma -s 3 -c 1 -o gpurun_out/prof_q1 -f python scripts/prof_driver.py q1 5 > gpurun_out/ncu_q1.log 2>&1; echo q1 rc=$?
 $NCU --set full --import-source on --clock-control none -k regex:q1n_ -s 3 -c 1 -o gpurun_out/prof_q1n -f python scripts/prof_driver.py q1n 5 > gpurun_out/ncu_q1n.log 2>&1; echo q1n rc=$?
 $NCU --set full --import-source on --clock-control none -k regex:select_fused -s 3 -c 1 -o gpurun_out/prof_rows -f python scripts/prof_driver.py rows 5 > gpurun_out/ncu_rows.log 2>&1; echo rows rc=$?
+$NCU --set full --import-source on --clock-control none -k regex:compact_kernel -s 3 -c 1 -o gpurun_out/prof_compact -f python scripts/prof_driver.py rows 5 > gpurun_out/ncu_compact.log 2>&1; echo compact rc=$?

@@ -10,4 +10,6 @@ timeout 900 $CS --tool memcheck --error-exitcode 9 python -m pytest tests/test_s
 timeout 900 $CS --tool racecheck --error-exitcode 9 python -m pytest tests/test_select_gpu.py -q -x -k "test_single_select_sizes_and_alignment" > gpurun_out/san_race_select.log 2>&1; echo select racecheck rc=$?
 timeout 900 $CS --tool racecheck --error-exitcode 9 python -m pytest tests/test_q1_gpu.py tests/test_q1_narrow_gpu.py -q -x -k "small_sizes or encode_matches" > gpurun_out/san_race_q1.log 2>&1; echo q1 racecheck rc=$?
 timeout 900 $CS --tool synccheck --error-exitcode 9 python -m pytest tests/test_select_gpu.py tests/test_select_multi_gpu.py -q -x -k "test_single_select_sizes_and_alignment or sizes_offsets" > gpurun_out/san_sync.log 2>&1; echo synccheck rc=$?
+timeout 900 $CS --tool memcheck --error-exitcode 9 python -m pytest tests/test_select_rows_gpu.py -q -x -k "phases or never_writes or both_payload" > gpurun_out/san_rows2.log 2>&1; echo rows2 memcheck rc=$?
+timeout 900 $CS --tool racecheck --error-exitcode 9 python -m pytest tests/test_select_rows_gpu.py -q -x -k "both_payload" > gpurun_out/san_race_rows.log 2>&1; echo rows racecheck rc=$?
 for f in gpurun_out/san_*.log; do echo "== $f"; grep -E "ERROR SUMMARY|passed|failed|Error" $f | tail -3; done

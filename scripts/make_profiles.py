@@ -26,6 +26,8 @@ CAPTURES = {  # report -> (summary name, traffic key, command)
     "prof_rows": ("select_rows_k2_s05_n28", "select_rows_k2_s0.5_n28",
                   "python scripts/prof_driver.py rows 5  (2^28 key + 2 int32 fields, k=2, s=0.5/stage)"),
     "prof_q1n": ("q1n_sf10", "q1n_sf10", "python scripts/prof_driver.py q1n 5  (SF10 narrow, 60M rows)"),
+    "prof_compact": ("compact_k2_s05_n28", "compact_k2_s0.5_n28",
+                     "python scripts/prof_driver.py rows 5  (payload compaction of 3 int32 fields, 2^28 rows, k=2, s=0.5/stage)"),
 }
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",

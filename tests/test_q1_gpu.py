@@ -90,6 +90,56 @@ def test_device_generated_sf10_launch_config(R):
     assert_same(rows, exp)
 
 
+def test_sf100_full_size_launch_config(R):
+    """BASELINE configs[4] at full size (SF100, 600 M rows, 22.8 GB on the
+    device, seed 5 as bench.py) in bench's launch configuration (one ra_q1 over
+    the whole table), plus the same rows as 4 row-range shards merged by
+    ra_q1_finalize (the N=4 exchange).  Expected values: the oracle over
+    50 M-row host chunks, exact sums added across chunks (partition
+    additivity, pinned in test_oracle_q1), AVG = the correctly rounded exact
+    quotient (C12)."""
+    from fractions import Fraction
+    from paper_conf_ipps_wudwcyc12_b200 import dist as rdist
+    sf, seed = 100, 5
+    n, parts = ragen.rows_for_sf(sf), ragen.parts_for_sf(sf)
+    dcols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+             for name, dt in ragen.LINEITEM_COLUMNS}
+    ragen.lineitem_dev(seed, parts, dcols)
+    rows, rc, part = gpu_q1(R, dcols)
+    assert rc == R.RA_OK and part.rows == n
+    shards = []
+    for r in range(4):
+        lo, hi = rdist.shard_range(n, r, 4)
+        p_ = R.q1({k: v[lo:hi] for k, v in dcols.items()})
+        shards.append(p_)
+    torch.cuda.synchronize()
+    srows, src = R.q1_finalize(b"".join(bytes(p_.cpu().numpy().tobytes()) for p_ in shards))
+    del dcols
+    tot = {}
+    chunk = 50_000_000
+    for lo in range(0, n, chunk):
+        m = min(chunk, n - lo)
+        part_rows, st = oracle.q1(ragen.lineitem(seed, m, parts, row0=lo), CUTOFF)
+        assert st == 0
+        for e in part_rows:
+            g = tot.setdefault((e["returnflag"], e["linestatus"]), dict.fromkeys(
+                ["count_order", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "sum_disc"], 0))
+            for k in g:
+                g[k] += e[k]
+    exp = []
+    for (rf, ls) in sorted(tot):
+        g = dict(tot[(rf, ls)], returnflag=rf, linestatus=ls)
+        c100 = 100 * g["count_order"]
+        g["avg_qty"] = float(Fraction(g["sum_qty"], c100))
+        g["avg_price"] = float(Fraction(g["sum_base_price"], c100))
+        g["avg_disc"] = float(Fraction(g["sum_disc"], c100))
+        exp.append(g)
+    assert sum(g["sum_charge"] for g in exp) > 2**63  # SF100: Sum(charge) needs more than int64 (C11)
+    assert_same(rows, exp)
+    assert src == R.RA_OK
+    assert_same(srows, exp)
+
+
 def test_domain_errors_reported(R):
     cols = ragen.lineitem(5, 50000, 2000)
     bad = {k: v.copy() for k, v in cols.items()}

@@ -418,7 +418,7 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     chains = [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)]]
     mo = [torch.empty(n, dtype=torch.int32, device=dev) for _ in range(2)]
     mc = torch.zeros(2, dtype=torch.int64, device=dev)
-    mws_b = R.ra_select_workspace_bytes(n, R.RA_MAX_PREDS, 1)
+    mws_b = R.ra_select_multi_workspace_bytes(n)
     mws = torch.zeros(mws_b, dtype=torch.uint8, device=dev)
     keepP = [R.make_preds(c) for c in chains]
     mch = (ctypes.c_void_p * 2)(*[ctypes.addressof(p_) for p_ in keepP])

@@ -211,9 +211,15 @@ int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h
  *  M             number of outputs, 1 <= M <= RA_MAX_OUTPUTS
  *  d_outs[o]     device int32[out_caps[o]]
  *  d_counts[o]   device int64: output o's size (the required size)
- *  d_ws          ra_select_workspace_bytes(n, RA_MAX_PREDS, 1), zeroed once
- * Rows beyond out_caps[o] are not written (the count is still exact). */
+ *  d_ws          ra_select_multi_workspace_bytes(n) bytes (for M = 1:
+ *                ra_select_workspace_bytes(n, RA_MAX_PREDS, 1)), zeroed once;
+ *                beyond the select status words it holds per-CTA spill slots
+ *                for tiles whose two runs exceed the shared-memory ring
+ * Rows beyond out_caps[o] are not written (the count is still exact).
+ * RA_E_WORKSPACE if ws_bytes is too small. */
 #define RA_MAX_OUTPUTS 2
+
+size_t ra_select_multi_workspace_bytes(int64_t n);
 
 int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const* h_chains, const int* ks, int M,
                     int32_t* const* d_outs, const int64_t* out_caps, int64_t* const* d_counts, void* d_ws,

@@ -23,7 +23,8 @@ from ._ra import (RA_E_CAPACITY, RA_E_DOMAIN, RA_OK, RA_Q1_GROUPS, make_preds, r
                   ra_q1_fission_run, ra_q1_fission_workspace_bytes, ra_q1_row, ra_q1_workspace_bytes,
                   ra_select_chain, ra_select_workspace_bytes, ra_lineitem_narrow, ra_lineitem_narrow_out,
                   ra_q1_encode, ra_q1_narrow, ra_q1_narrow_fission_run, ra_q1_narrow_fission_workspace_bytes,
-                  ra_payload, ra_select_rows, ra_select_rows_workspace_bytes, ra_select_multi, RA_MAX_PREDS)
+                  ra_payload, ra_select_rows, ra_select_rows_workspace_bytes, ra_select_multi, RA_MAX_PREDS,
+                  ra_select_multi_workspace_bytes)
 
 Q1_CUTOFF_DELTA90 = 10471  # 1998-12-01 - 90 days = 1998-09-02
 LINEITEM_COLUMNS = ("shipdate", "returnflag", "linestatus", "quantity", "extendedprice", "discount", "tax")
@@ -98,7 +99,7 @@ def select_multi(x, chains, outs=None, stream=None):
     op = (ctypes.c_void_p * M)(*[o.data_ptr() for o in outs])
     caps = (ctypes.c_int64 * M)(*[o.numel() for o in outs])
     cp = (ctypes.c_void_p * M)(*[counts.data_ptr() + 8 * o for o in range(M)])
-    ws = workspace(x.device, "select_fused", ra_select_workspace_bytes(n, RA_MAX_PREDS, 1), stream)
+    ws = workspace(x.device, "select_fused", ra_select_multi_workspace_bytes(n), stream)
     ra_select_multi(x.data_ptr(), n, ch, ks, M, op, caps, cp, ws.data_ptr(), ws.numel(), _stream_handle(stream))
     return outs, counts
 

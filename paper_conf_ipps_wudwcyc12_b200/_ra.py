@@ -122,6 +122,7 @@ _SIGS = {
     "ra_select_chain": ([_vp, _i64, _vp, _i32, _i32, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_select_multi": ([_vp, _i64, _vp, _vp, _i32, _vp, _vp, _vp, _vp, _sz, _vp], _i32),
     "ra_select_rows_workspace_bytes": ([_i64, _i32], _sz),
+    "ra_select_multi_workspace_bytes": ([_i64], _sz),
     "ra_select_rows": ([_vp, _i64, _vp, _i32, _vp, _vp, _i32, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_q1_workspace_bytes": ([_i64], _sz),
     "ra_q1": ([_vp, _i64, ctypes.c_int32, _vp, _vp, _sz, _vp], _i32),
@@ -188,6 +189,10 @@ def ra_select_chain(d_in: int, n: int, h_preds, k: int, fused: int, d_out: int, 
 def ra_select_multi(d_in: int, n: int, h_chains, ks, M: int, d_outs, out_caps, d_counts, d_ws: int,
                     ws_bytes: int, stream: int) -> None:
     _check(_lib.ra_select_multi(d_in, n, h_chains, ks, M, d_outs, out_caps, d_counts, d_ws, ws_bytes, stream))
+
+
+def ra_select_multi_workspace_bytes(n: int) -> int:
+    return int(_lib.ra_select_multi_workspace_bytes(n))
 
 
 def ra_select_rows_workspace_bytes(n: int, k: int) -> int:

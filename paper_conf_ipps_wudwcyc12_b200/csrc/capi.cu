@@ -178,6 +178,11 @@ RA_API int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_pred
                            (cudaStream_t)stream);
 }
 
+RA_API size_t ra_select_multi_workspace_bytes(int64_t n) {
+  if (n < 0) n = 0;
+  return ((ra_select_workspace_bytes(n, RA_MAX_PREDS, 1) + 255) / 256) * 256 + ra::sel_spill_bytes(n);
+}
+
 RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const* h_chains, const int* ks, int M,
                            int32_t* const* d_outs, const int64_t* out_caps, int64_t* const* d_counts, void* d_ws,
                            size_t ws_bytes, ra_stream_t stream) {
@@ -203,6 +208,9 @@ RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const*
   second.out = d_outs[1];
   second.out_cap = out_caps[1];
   second.d_count = d_counts[1];
+  const size_t need = ra_select_multi_workspace_bytes(n);
+  if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
+  second.spill = (int32_t*)((char*)d_ws + ((ra_select_workspace_bytes(n, RA_MAX_PREDS, 1) + 255) / 256) * 256);
   return launch_select_pass(d_in, n, nullptr, cp[0], d_outs[0], out_caps[0], d_counts[0], d_ws, (cudaStream_t)stream,
                             nullptr, &second);
 }

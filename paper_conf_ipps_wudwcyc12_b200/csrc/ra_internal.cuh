@@ -69,7 +69,10 @@ struct SelSecond {
   int32_t* out;
   int64_t out_cap;
   int64_t* d_count;
+  int32_t* spill;  // sel_spill_bytes(n) of workspace (second runs the ring cannot hold)
 };
+constexpr int SEL_MULTI_MAX_GRID = 320;  // CTAs of a two-output pass (>= 2 per SM on 148 SMs)
+size_t sel_spill_bytes(int64_t n);
 // Row-id mode extras for the payload compaction (compact.cu), per select tile t
 // (SEL_TILE rows counted from the key's 16-B aligned base): the compute lanes'
 // flag words fmask[t*SEL_THREADS + tid] and a 48-B record meta[t*12 ..]: the

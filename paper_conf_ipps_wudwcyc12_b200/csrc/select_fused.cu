@@ -153,6 +153,7 @@ struct SelParams {
   int32_t n_ne2;
   int32_t ne2[RA_MAX_PREDS];
   int32_t* out2;
+  int32_t* spill;  // M == 2: per-CTA global slots [K][SEL_TILE] for second runs the ring cannot hold
   int64_t out_cap2;
   int64_t* d_count2;
   int32_t lo;
@@ -181,17 +182,17 @@ struct __align__(128) SelSmemT {
   int32_t cnt2[K];                     // M == 2: second output's tile aggregates (run after the first)
   int64_t goff2[K];                    // M == 2: second output's tile offsets
   int32_t start[K];                    // tile run start in the ring
+  int32_t spilled[K];                  // M == 2: the tile's second run is in its spill slot
   int64_t n;
   uint32_t epoch;
   int32_t demand;  // oldest tile the compute warps are waiting to write (-1: none yet)
 };
-// One output: a 40 KB ring (2 CTAs/SM).  Two outputs (ra_select_multi): a
-// tile's two runs together hold up to 2 x 8192 rows, so the ring doubles
-// (1 CTA/SM).
+// A 40 KB ring (2 CTAs/SM), also for two outputs (ra_select_multi): a tile
+// whose two runs exceed it is placed straight from registers (the compute
+// loop's "direct" path).
 using SelSmem = SelSmemT<SEL_OUTRING>;
-using SelSmem2 = SelSmemT<2 * SEL_TILE>;
 template <int M>
-using SmemFor = typename std::conditional<M == 2, SelSmem2, SelSmem>::type;
+using SmemFor = SelSmem;
 
 using dev::smem_u32;
 using dev::mbar_init;
@@ -251,6 +252,19 @@ __device__ __forceinline__ int32_t comp(const int4& v, int c) {
 }
 
 // Store v at shared byte address a and advance a, iff (fl & mask) != 0.
+// The same into global memory (M == 2 spill slots).
+__device__ __forceinline__ void put_if_global(int32_t*& a, uint32_t fl, uint32_t mask, int32_t v) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\t.reg .b32 t;\n\t"
+      "and.b32 t, %1, %2;\n\t"
+      "setp.ne.u32 q, t, 0;\n\t"
+      "@q st.global.b32 [%0], %3;\n\t"
+      "@q add.u64 %0, %0, 4;\n\t}"
+      : "+l"(a)
+      : "r"(fl), "r"(mask), "r"(v)
+      : "memory");
+}
+
 __device__ __forceinline__ void put_if(uint32_t& a, uint32_t fl, uint32_t mask, int32_t v) {
   asm volatile(
       "{\n\t.reg .pred q;\n\t.reg .b32 t;\n\t"
@@ -391,7 +405,12 @@ __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int
     int64_t lim2 = P.out_cap2 - g2;
     lim2 = lim2 < 0 ? 0 : (lim2 > c2 ? c2 : lim2);
     int32_t* __restrict__ out2 = P.out2 + g2;
-    for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = run[c + e];
+    if (S.spilled[k % K]) {  // from the spill slot (global, L2)
+      const int32_t* sp = P.spill + ((int64_t)blockIdx.x * K + k % K) * SEL_TILE;
+      for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = sp[e];
+    } else {
+      for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = run[c + e];
+    }
   }
   if (!ROWS) {
     int32_t* __restrict__ out = P.out + g;
@@ -665,9 +684,15 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       agg2 = (int32_t)__reduce_add_sync(0xffffffffu, wt2);
       wbase2 = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt2 : 0u);
     }
+    // M == 2: when both runs together exceed the ring (both outputs keep most
+    // of the tile), the second run goes to this CTA's global spill slot for
+    // the tile (read back when the tile is written).  Measured: spilling both
+    // runs, or placing such tiles straight from registers after waiting for
+    // their own placement, is slower still.
+    const bool spill2 = M == 2 && agg + agg2 > RING;
     if (ROWS && P.meta && lane == 0) P.meta[t * 12 + warp] = (uint32_t)wbase;
     const bool ring_rows = !ROWS || P.rowids;  // ROWS without ids: placement only, no ring
-    const int32_t rows_in = ring_rows ? agg + agg2 : 0;  // ring rows this tile needs (both runs)
+    const int32_t rows_in = ring_rows ? agg + (spill2 ? 0 : agg2) : 0;  // ring rows this tile needs
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
       mbar_arrive(&S.empty[slot]);  // input slot free: the producer refills it
       const uint64_t aggw = M == 2 ? ((uint64_t)agg | ((uint64_t)agg2 << 16)) : (uint64_t)agg;
@@ -680,7 +705,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ---- allocate the tile's run: contiguous in the ring (a run that does not
     // fit before the end starts again at 0); write the oldest tiles early if
     // the ring is short.  Every thread takes the same decisions.
-    int32_t start;
+    int32_t start = 0;
     bool forced = false;
     while (true) {
       if (used == 0) {  // nothing pending (or only empty runs)
@@ -698,12 +723,15 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         break;
       }
       write_tile<ROWS, M, SM>(S, P, head, tid);
-      used -= ring_rows ? S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0) : 0;
+      used -= ring_rows ? S.cnt[head % K] + (M == 2 && !S.spilled[head % K] ? S.cnt2[head % K] : 0) : 0;
       ++head;
       forced = true;
     }
     if (forced) compute_bar();  // rows written out are read before they are overwritten
-    if (tid == 0) S.start[i % K] = start;
+    if (tid == 0) {
+      S.start[i % K] = start;
+      if (M == 2) S.spilled[i % K] = spill2;
+    }
     used += rows_in;
     // ---- scatter the tile into the ring (M == 2: the second run after the first)
 #pragma unroll
@@ -713,6 +741,19 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
 #if RA_SEL_PTXSCATTER
       const uint32_t ring0 = smem_u32(S.ring);
 #endif
+      if (M == 2 && o == 1 && spill2) {  // second run -> the tile's spill slot (global)
+        int32_t* slot = P.spill + ((int64_t)blockIdx.x * K + i % K) * SEL_TILE;
+        rb = wbase2;
+#pragma unroll
+        for (int j = 0; j < SEL_VEC; ++j) {
+          const int q = NPK * o + q_of(j);
+          int32_t* a = slot + rb + (int32_t)(((inc[q] - packed[q]) >> (8 * b_of(j))) & 0xFFu);
+#pragma unroll
+          for (int c = 0; c < 4; ++c) put_if_global(a, f, 1u << (4 * j + c), comp(v[j], c));
+          rb += (int32_t)((tot[q] >> (8 * b_of(j))) & 0xFFu);
+        }
+        continue;
+      }
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
         const int q = NPK * o + q_of(j);
@@ -742,7 +783,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ---- gather: tile i - LAG is due
     if (i - LAG >= head) {
       write_tile<ROWS, M, SM>(S, P, head, tid);
-      used -= ring_rows ? S.cnt[head % K] + (M == 2 ? S.cnt2[head % K] : 0) : 0;
+      used -= ring_rows ? S.cnt[head % K] + (M == 2 && !S.spilled[head % K] ? S.cnt2[head % K] : 0) : 0;
       ++head;
     }
   }
@@ -785,6 +826,12 @@ int64_t sel_max_tiles(int64_t n) { return (n + 3 + SEL_TILE - 1) / SEL_TILE + 1;
 
 size_t sel_status_bytes(int64_t n) { return SEL_HDR_BYTES + 8 * (size_t)sel_max_tiles(n) + 16; }
 
+size_t sel_spill_bytes(int64_t n) {
+  int64_t g = sel_max_tiles(n);
+  if (g > SEL_MULTI_MAX_GRID) g = SEL_MULTI_MAX_GRID;
+  return (size_t)g * K * SEL_TILE * 4;
+}
+
 size_t sel_inter_bytes(int64_t n) {
   // two int32[n] relations + two int64 counts, 256-B granules
   const size_t rel = (((size_t)(n > 0 ? n : 1) * 4 + 255) / 256) * 256;
@@ -812,6 +859,7 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   P.n_ne2 = 0;
   for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne2[j] = 0;
   P.out2 = nullptr;
+  P.spill = nullptr;
   P.out_cap2 = 0;
   P.d_count2 = nullptr;
   if (second) {
@@ -827,6 +875,7 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
       P.ne2[0] = 0;
     }
     P.out2 = second->out;
+    P.spill = second->spill;
     P.out_cap2 = second->out_cap;
     P.d_count2 = second->d_count;
   }
@@ -875,13 +924,14 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   if (rc) return rc;
   const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
   int64_t grid = (int64_t)num_sms() * per_sm;
+  if (two && grid > SEL_MULTI_MAX_GRID) grid = SEL_MULTI_MAX_GRID;  // spill slots exist for this many CTAs
   if (grid > ntiles_max) grid = ntiles_max;
   if (grid < 1) grid = 1;
   // No co-residency is required (plain launch): a CTA only ever waits on the
   // aggregates of tiles with lower tickets, tickets are drawn only by running
   // CTAs, and a tile's aggregate is published before its CTA can block on
   // any placement — so the lowest unpublished tile can always be published.
-  const size_t smem = two ? sizeof(SelSmem2) : sizeof(SelSmem);
+  const size_t smem = sizeof(SelSmem);
   void* args[] = {(void*)&P};
 #if RA_SEL_COOP
   cudaError_t le = cudaLaunchCooperativeKernel(kern, dim3((unsigned)grid), dim3(BLOCK), args, smem, s);

@@ -88,6 +88,38 @@ def test_capacity(R):
     assert np.array_equal(outs[1][:e1.size].cpu().numpy(), e1)
 
 
+@pytest.mark.parametrize("caps", [(1000, 5), (3 * 8192 + 17, 10**9), (0, 123457)])
+def test_capacity_dense_outputs(R, caps):
+    """Both outputs keep ~90% of every tile, more than the selected-row ring
+    holds: those tiles are placed straight from registers; truncation stays exact
+    and nothing is written past either capacity."""
+    n = 50 * 8192 + 99
+    x = ragen.int32_column(76, n)
+    xd = torch.from_numpy(x).cuda()
+    chains = [[("lt", ragen.nested_thresholds(0.9, 1)[0])], [("gt", -ragen.nested_thresholds(0.9, 1)[0])]]
+    e0, e1 = oracle.select_multi(x, chains)
+    cap = [min(c, n) for c in caps]
+    outs = [torch.full((c + 64,), -3, dtype=torch.int32, device="cuda") for c in cap]
+    P = [R.make_preds(c) for c in chains]
+    import ctypes
+    mch = (ctypes.c_void_p * 2)(*[ctypes.addressof(p_) for p_ in P])
+    mks = (ctypes.c_int * 2)(1, 1)
+    mop = (ctypes.c_void_p * 2)(*[o.data_ptr() for o in outs])
+    mcap = (ctypes.c_int64 * 2)(*cap)
+    cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+    mcp = (ctypes.c_void_p * 2)(cnt.data_ptr(), cnt.data_ptr() + 8)
+    wsb = R.ra_select_multi_workspace_bytes(n)
+    ws = torch.zeros(wsb, dtype=torch.uint8, device="cuda")
+    R.ra_select_multi(xd.data_ptr(), n, mch, mks, 2, mop, mcap, mcp, ws.data_ptr(), wsb, 0)
+    torch.cuda.synchronize()
+    assert [int(v) for v in cnt.cpu().tolist()] == [e0.size, e1.size]
+    for o, e, c in zip(outs, (e0, e1), cap):
+        h = o.cpu().numpy()
+        m = min(c, e.size)
+        assert np.array_equal(h[:m], e[:m])
+        assert (h[m:] == -3).all()
+
+
 def test_argument_errors(R):
     xd = torch.zeros(16, dtype=torch.int32, device="cuda")
     with pytest.raises(R.RAError) as e:

@@ -24,10 +24,10 @@ namespace {
 
 constexpr int CT_WARPS = SEL_THREADS / 32;   // compute warps = select warps per tile (8)
 constexpr int CT_BLOCK = SEL_THREADS + 32;   // + the producer warp
-constexpr int SLICE = SEL_TILE / CT_WARPS;   // rows per warp slice (1024)
+constexpr int CT_SLICE = SEL_TILE / CT_WARPS;   // rows per warp slice (1024)
 constexpr int CT_STAGES = 3;  // x 2 CTAs per SM
-constexpr int STAGE_BYTES = SEL_TILE * 4;    // one tile of a 4-byte field, half a tile of an 8-byte one
-static_assert(SLICE == 32 * SEL_VEC * 4, "a slice is 32 lanes x SEL_VEC vectors x 4 rows");
+constexpr int CT_STAGE_BYTES = SEL_TILE * 4;    // one tile of a 4-byte field, half a tile of an 8-byte one
+static_assert(CT_SLICE == 32 * SEL_VEC * 4, "a slice is 32 lanes x SEL_VEC vectors x 4 rows");
 
 struct CompactParams {
   const uint32_t* fmask;  // [tile][SEL_THREADS] flag words
@@ -45,7 +45,7 @@ struct CompactParams {
 };
 
 struct __align__(128) CtSmem {
-  int4 data[CT_STAGES][STAGE_BYTES / 16];
+  int4 data[CT_STAGES][CT_STAGE_BYTES / 16];
   uint32_t fl[CT_STAGES][SEL_THREADS];
   uint32_t meta[CT_STAGES][12];
   uint64_t full[CT_STAGES];
@@ -142,7 +142,7 @@ __device__ __forceinline__ void place(const CompactParams& P, int f, const int4*
     for (int u = 0; u < G; ++u) {
       const int j = j0 + u;
       int32_t p = rb + (int32_t)((ex[j & 1] >> (8 * (j >> 1))) & 0xFFu);
-      if (lim >= SLICE) {  // the whole slice fits: one predicated store + add per row
+      if (lim >= CT_SLICE) {  // the whole slice fits: one predicated store + add per row
         T* a = out + p;
 #pragma unroll
         for (int c = 0; c < 4; ++c) put_if_global(a, fl, 1u << (4 * j + c), e[u][c]);
@@ -221,13 +221,13 @@ __global__ void __launch_bounds__(CT_BLOCK, 2) compact_kernel(const CompactParam
       // 8-byte fields: unit h holds slices 4h..4h+3 (warps 4h..4h+3)
       const bool mine = P.eb[f] == 4 || (warp >> 2) == h;
       if (mine && __any_sync(0xffffffffu, fl != 0u) && dst0 < cnt) {
-        const int32_t lim = cnt - dst0 < SLICE ? (int32_t)(cnt - dst0) : SLICE;
+        const int32_t lim = cnt - dst0 < CT_SLICE ? (int32_t)(cnt - dst0) : CT_SLICE;
         uint32_t ex[2], tot[2];
         packed_scan(fl, lane, ex, tot);
         // the warp's slice in the staged unit
         const int4* tile = !P.vec[f] ? nullptr
-                           : P.eb[f] == 4 ? &S.data[s][warp * (SLICE / 4)] : &S.data[s][(warp & 3) * (SLICE / 2)];
-        const int64_t vbase = t * SEL_TILE + warp * SLICE;
+                           : P.eb[f] == 4 ? &S.data[s][warp * (CT_SLICE / 4)] : &S.data[s][(warp & 3) * (CT_SLICE / 2)];
+        const int64_t vbase = t * SEL_TILE + warp * CT_SLICE;
         if (P.eb[f] == 4)
           place<uint32_t>(P, f, tile, lane, vbase, fl, dst0, lim, ex, tot);
         else
@@ -246,7 +246,7 @@ __global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ f
   const int64_t cnt = *d_count;
   if (cnt * sparse_den > n) return;  // dense: compact_kernel places the fields, no ids needed
   const int lane = threadIdx.x & 31;
-  const int64_t nslices = (n + mis + SLICE - 1) / SLICE;
+  const int64_t nslices = (n + mis + CT_SLICE - 1) / CT_SLICE;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
   const int64_t w0 = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
   constexpr int U = 4;  // slices per warp iteration: their loads are issued together
@@ -267,7 +267,7 @@ __global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ f
       if (!__any_sync(0xffffffffu, fl[q] != 0u)) continue;
       uint32_t ex[2], tot[2];
       packed_scan(fl[q], lane, ex, tot);
-      const uint32_t r0 = (uint32_t)((sb + q) * SLICE - mis);  // row of the slice's first virtual row (mod 2^32)
+      const uint32_t r0 = (uint32_t)((sb + q) * CT_SLICE - mis);  // row of the slice's first virtual row (mod 2^32)
       uint32_t* a0 = ids + dst0[q];
       int32_t rb = 0;
 #pragma unroll
@@ -287,7 +287,7 @@ int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, c
                           int32_t sparse_den, uint32_t* ids, cudaStream_t s) {
   if (n == 0) return RA_OK;
   const int32_t mis = (int32_t)(((uintptr_t)d_key & 15u) >> 2);
-  const int64_t nslices = (n + mis + SLICE - 1) / SLICE;
+  const int64_t nslices = (n + mis + CT_SLICE - 1) / CT_SLICE;
   int64_t grid = (nslices + 31) / 32;  // 8 warps x 4 slices per CTA iteration
   const int64_t lim = (int64_t)num_sms() * 8;
   if (grid > lim) grid = lim;

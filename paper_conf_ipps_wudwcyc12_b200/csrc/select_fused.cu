@@ -466,7 +466,9 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       // as the current one starts, so an atomic's L2 round trip overlaps G
       // tiles of work.  G = 1 (measured, 2^28 rows: G = 2 is 2-4% faster at
       // overall selectivity <= .25 but 40% slower at .5/.9, where a drawn,
-      // not yet counted tile holds up every later tile's placement).
+      // not yet counted tile holds up every later tile's placement; a second
+      // single ticket drawn ahead only while the ring is under half full
+      // gained nothing at .01/.25 and lost 5% at .5).
       constexpr int G = RA_SEL_BATCH;
       int64_t cur = (int64_t)atomicAdd(P.ticket, (unsigned long long)G);
       int64_t nxt = 0;

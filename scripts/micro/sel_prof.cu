@@ -7,6 +7,7 @@
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/q1_fused.cu"
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/q1_narrow.cu"
 #include "../../paper_conf_ipps_wudwcyc12_b200/csrc/gather.cu"
+#include "../../paper_conf_ipps_wudwcyc12_b200/csrc/compact.cu"
 #include <cstdlib>
 #ifndef VARIANT
 #define VARIANT "full"

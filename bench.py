@@ -314,6 +314,7 @@ def run_ours(args, D: Dist):
 
 def extras(args, D, torch, R, x, preds, kept, chain_ms):
     """Other BASELINE configs + e2e + CPU baseline, same timing rules."""
+    from paper_conf_ipps_wudwcyc12_b200 import dist as rdist
     s_sel = args.sel
     dev = x.device
     sh = int(torch.cuda.current_stream().cuda_stream)
@@ -412,6 +413,35 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                             "h2d_bytes_per_step": 4 * n3, "d2h_bytes_per_step": 4 * k3 + 8 * (n3 >> 24),
                             "pcie_h2d_gbs": 4 * n3 / (f3ms * 1e-3) / 1e9}
         del h3, o3
+
+    # --- d5 shape for SELECT: 2^30 device-resident rows split across the ranks
+    # (strong scaling), fused k-chain + the count exchange
+    nb = (1 << 30) // D.world
+    xb = torch.empty(nb, dtype=torch.int32, device=dev)
+    ragen.int32_column_dev(CHAIN_SEED + 200, xb, row0=D.rank * nb, stream=sh)
+    ob = torch.empty(nb, dtype=torch.int32, device=dev)
+    cb = torch.zeros(1, dtype=torch.int64, device=dev)
+    wsb_b = R.ra_select_workspace_bytes(nb, k, 1)
+    wsb = torch.zeros(wsb_b, dtype=torch.uint8, device=dev)
+    Pb = R.make_preds(preds)
+    ab = (xb.data_ptr(), nb, Pb, k, 1, ob.data_ptr(), nb, cb.data_ptr(), wsb.data_ptr(), wsb_b, sh)
+
+    def big_step(i, kernel_done=False):
+        if not kernel_done:
+            R.ra_select_chain(*ab)
+        if D.pg:
+            rdist.exchange_counts(cb)
+
+    bms, bkms = timed(torch, D, big_step, 20, 3, kernel_fn=lambda i: R.ra_select_chain(*ab))
+    bk = int(cb.item())
+    bach = (4 * nb + 4 * bk) / (bkms * 1e-3) / 1e9
+    ex["select_1g_device"] = {"workload": f"2^30 int32 rows device-resident, split over {D.world} rank(s), k={k}, "
+                                          f"s={s_sel}/stage (SURVEY d5 shape)",
+                              "rows": 1 << 30, "rows_per_s": (1 << 30) / (bms * 1e-3), "ms_per_step": bms,
+                              "kernel_ms": bkms, "scaling": "strong",
+                              "roofline": {"kernel": "select_fused_kernel", "bound": "hbm", "achieved": bach,
+                                           "peak": peak, "unit": "GB/s", "frac": bach / peak}}
+    del xb, ob, wsb
 
     # --- f2: two SELECTs filtering the same input (Fig 2(c)): one fused pass
     # vs the two SELECT kernels run one after the other (two input reads)

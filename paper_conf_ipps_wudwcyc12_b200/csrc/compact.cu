@@ -161,6 +161,7 @@ __device__ __forceinline__ void place(const CompactParams& P, int f, const int4*
 }
 
 __global__ void __launch_bounds__(CT_BLOCK, 2) compact_kernel(const CompactParams P) {
+  dev::grid_dep_wait();
   extern __shared__ __align__(128) unsigned char smem_raw[];
   CtSmem& S = *reinterpret_cast<CtSmem*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -243,6 +244,7 @@ __global__ void __launch_bounds__(CT_BLOCK, 2) compact_kernel(const CompactParam
 __global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ fmask, const uint32_t* __restrict__ meta,
                                                   const int64_t* __restrict__ d_count, int64_t n, int32_t mis,
                                                   int32_t sparse_den, uint32_t* __restrict__ ids) {
+  dev::grid_dep_wait();
   const int64_t cnt = *d_count;
   if (cnt * sparse_den > n) return;  // dense: compact_kernel places the fields, no ids needed
   const int lane = threadIdx.x & 31;
@@ -291,9 +293,9 @@ int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, c
   int64_t grid = (nslices + 31) / 32;  // 8 warps x 4 slices per CTA iteration
   const int64_t lim = (int64_t)num_sms() * 8;
   if (grid > lim) grid = lim;
-  ids_kernel<<<(unsigned)grid, 256, 0, s>>>(mk.fmask, mk.meta, d_count, n, mis, sparse_den, ids);
+  cudaError_t e = launch_pdl(ids_kernel, dim3((unsigned)grid), dim3(256), 0, s, (const uint32_t*)mk.fmask,
+                             (const uint32_t*)mk.meta, d_count, n, mis, sparse_den, ids);
   count_launch();
-  cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "ids_kernel launch");
   return RA_OK;
 }
@@ -334,9 +336,8 @@ int launch_compact(const int32_t* d_key, int64_t n, const SelMasks& mk, const in
   const int64_t ntiles = (n + P.mis + SEL_TILE - 1) / SEL_TILE;
   int64_t grid = (int64_t)num_sms() * 2;  // 2 CTAs per SM (launch bounds, ~100 KB of ring each)
   if (grid > ntiles) grid = ntiles;
-  compact_kernel<<<(unsigned)grid, CT_BLOCK, sizeof(CtSmem), s>>>(P);
+  cudaError_t e = launch_pdl(compact_kernel, dim3((unsigned)grid), dim3(CT_BLOCK), sizeof(CtSmem), s, P);
   count_launch();
-  cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "compact_kernel launch");
   return RA_OK;
 }

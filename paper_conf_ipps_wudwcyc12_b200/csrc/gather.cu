@@ -23,6 +23,7 @@ constexpr int GATHER_U = 4;
 __global__ void __launch_bounds__(GATHER_T) gather_kernel(const uint32_t* __restrict__ ids,
                                                           const int64_t* __restrict__ d_count, int64_t cap,
                                                           const GatherSpec g) {
+  dev::grid_dep_wait();
   int64_t cnt = *d_count;
   if (cnt * g.sparse_den > g.n) return;  // dense: compact_kernel places the fields
   if (cnt > cap) cnt = cap;
@@ -72,9 +73,8 @@ int launch_gather(const uint32_t* ids, const int64_t* d_count, int64_t cap, cons
   int64_t grid = (cap + GATHER_T * GATHER_U - 1) / (GATHER_T * GATHER_U);
   const int64_t lim = (int64_t)num_sms() * 8;
   if (grid > lim) grid = lim;
-  gather_kernel<<<(unsigned)grid, GATHER_T, 0, s>>>(ids, d_count, cap, g);
+  cudaError_t e = launch_pdl(gather_kernel, dim3((unsigned)grid), dim3(GATHER_T), 0, s, ids, d_count, cap, g);
   count_launch();
-  cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "gather_kernel launch");
   return RA_OK;
 }

@@ -177,6 +177,7 @@ __device__ __forceinline__ void process_group(Acc& A, const Group4& G, int32_t c
 }
 
 __global__ void __launch_bounds__(Q1G_THREADS, 2) q1_grid_kernel(const Q1Params P) {
+  dev::grid_dep_wait();  // launch_pdl: the previous kernel's writes (e.g. a running partial) are visible
   __shared__ uint64_t s_w[Q1G_THREADS / 32][NS][8];
   __shared__ uint32_t s_status;
   __shared__ bool s_last;
@@ -321,6 +322,7 @@ __device__ __forceinline__ void flush(NarrowAcc& A, Q1TmaSmem& S, int tid) {
 }
 
 __global__ void __launch_bounds__(Q1T_NT + 32, 1) q1_tma_kernel(const Q1Params P) {
+  dev::grid_dep_wait();  // launch_pdl: the previous kernel's writes (e.g. a running partial) are visible
   extern __shared__ __align__(128) unsigned char q1_smem_raw[];
   Q1TmaSmem& S = *reinterpret_cast<Q1TmaSmem*>(q1_smem_raw);
   const int tid = threadIdx.x;
@@ -487,9 +489,8 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
     const int64_t min_grid = (n >> 17) / Q1T_NT + 1;
     if (grid < min_grid) grid = min_grid;
     if (grid > Q1_MAX_GRID) return fail(RA_E_INVAL, "n too large for the Q1 grid");
-    q1_tma_kernel<<<(unsigned)grid, Q1T_NT + 32, Q1T_SMEM, s>>>(P);
+    cudaError_t e = launch_pdl(q1_tma_kernel, dim3((unsigned)grid), dim3(Q1T_NT + 32), Q1T_SMEM, s, P);
     count_launch();
-    cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "q1_tma_kernel launch");
     return RA_OK;
   }
@@ -513,9 +514,8 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
   if (grid < min_grid) grid = min_grid;
   if (grid < 1) grid = 1;
   if (grid > Q1_MAX_GRID) return fail(RA_E_INVAL, "n too large for the Q1 grid");
-  q1_grid_kernel<<<(unsigned)grid, Q1G_THREADS, 0, s>>>(P);
+  cudaError_t e = launch_pdl(q1_grid_kernel, dim3((unsigned)grid), dim3(Q1G_THREADS), 0, s, P);
   count_launch();
-  cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "q1_grid_kernel launch");
   return RA_OK;
 }

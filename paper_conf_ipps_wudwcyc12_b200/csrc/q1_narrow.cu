@@ -163,6 +163,7 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
 }
 
 __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const QnParams P) {
+  dev::grid_dep_wait();  // launch_pdl: the previous kernel's writes (e.g. a running partial) are visible
   extern __shared__ __align__(128) unsigned char qn_smem_raw[];
   QnSmem& S = *reinterpret_cast<QnSmem*>(qn_smem_raw);
   const int tid = threadIdx.x;
@@ -327,9 +328,8 @@ int launch_q1_narrow(const ra_lineitem_narrow& c, int64_t n, int32_t cutoff, ra_
   const int64_t min_grid = (n >> 24) + 1;
   if (grid < min_grid) grid = min_grid;
   if (grid > Q1_MAX_GRID) return fail(RA_E_INVAL, "n too large for the Q1 grid");
-  q1n_kernel<<<(unsigned)grid, QN_NT + 32, QN_SMEM, s>>>(P);
+  cudaError_t e = launch_pdl(q1n_kernel, dim3((unsigned)grid), dim3(QN_NT + 32), QN_SMEM, s, P);
   count_launch();
-  cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "q1n_kernel launch");
   return RA_OK;
 }

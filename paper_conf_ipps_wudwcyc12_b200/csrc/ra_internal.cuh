@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <utility>
 
 #include "ra.h"
 
@@ -22,6 +23,23 @@ extern std::atomic<uint64_t> g_launches;
 inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
 
 int num_sms();  // of the current device (cached per device)
+
+// Launch with programmatic stream serialization (see dev::grid_dep_wait).
+template <typename... Params, typename... Args>
+cudaError_t launch_pdl(void (*kern)(Params...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                       Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 // ------------------------------------------------- predicate canonical form
 // A conjunction of k (op, value) predicates on a signed int32 equals
@@ -175,6 +193,12 @@ __device__ __forceinline__ uint32_t atom_add_acq_rel_u32(uint32_t* p, uint32_t v
   asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
   return old;
 }
+
+// ---- programmatic dependent launch: a kernel launched by launch_pdl may start
+// while the previous kernel on the stream finishes; it calls grid_dep_wait()
+// before its first global-memory access (the previous grid's writes are then
+// visible).
+__device__ __forceinline__ void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
 // ---- mbarrier + bulk-copy (TMA engine) helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {

@@ -99,8 +99,8 @@ constexpr int BLOCK = SEL_THREADS + 64;  // + the look-back and producer warps
 #endif
 constexpr int LAG = RA_SEL_LAG;          // tile k is written when tile k+LAG is counted (or earlier)
 constexpr int K = LAG + 2;               // metadata slots: tiles counted but not yet written
-#ifndef RA_SEL_COOP
-#define RA_SEL_COOP 0
+#ifndef RA_SEL_PDL
+#define RA_SEL_PDL 1
 #endif
 #ifndef RA_SEL_PTXSCATTER
 #define RA_SEL_PTXSCATTER 1
@@ -430,6 +430,11 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
   SM& S = *reinterpret_cast<SM*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
+  // Programmatic dependent launch (launch_select_pass): this grid may start
+  // while the previous kernel on the stream is finishing.  Nothing here reads
+  // or writes global memory before the wait: the previous grid's results (its
+  // output, count, epoch bump and ticket reset) are visible after it.
+  dev::grid_dep_wait();
   if (tid == 0) {
     int64_t n = P.n;
     if (P.d_n) {
@@ -935,11 +940,17 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   // any placement — so the lowest unpublished tile can always be published.
   const size_t smem = sizeof(SelSmem);
   void* args[] = {(void*)&P};
-#if RA_SEL_COOP
-  cudaError_t le = cudaLaunchCooperativeKernel(kern, dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
-#else
-  cudaError_t le = cudaLaunchKernel(kern, dim3((unsigned)grid), dim3(BLOCK), args, smem, s);
-#endif
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(BLOCK);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;  // overlap this launch with the previous
+  attr[0].val.programmaticStreamSerializationAllowed = RA_SEL_PDL;   // kernel's tail (griddepcontrol.wait)
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t le = cudaLaunchKernelExC(&cfg, kern, args);
   if (le != cudaSuccess) return cuda_fail(le, "select_fused_kernel launch");
   count_launch();
   return RA_OK;

@@ -114,7 +114,10 @@ constexpr int K = LAG + 2;               // metadata slots: tiles counted but no
 #endif
 constexpr int D1 = RA_SEL_D1;            // window of tile k copied when tile k+D1 is counted
 constexpr int D2 = RA_SEL_D2;            // ... and resolved when tile k+D2 is counted
-constexpr int Q = D2 - D1 + 1;           // window slots
+#ifndef RA_SEL_Q
+#define RA_SEL_Q (RA_SEL_D2 - RA_SEL_D1 + 1)
+#endif
+constexpr int Q = RA_SEL_Q;              // window slots (windows in flight)
 constexpr int LBW = 10;                  // window words per lane per pass
 #ifndef RA_SEL_WIN
 #define RA_SEL_WIN 768

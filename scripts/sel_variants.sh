@@ -6,7 +6,7 @@ NV="/usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -linein
 for v in $V; do
   IFS=, read vec ah ring d1 d2 lag extra <<< "$v"
   tag=${vec}_${ah}_${ring}_${d1}_${d2}_${lag}${extra:+_$extra}
-  ex=${extra:+-D$extra}
+  ex=${extra:+-D${extra//+/ -D}}
   b=scripts/micro/selv_$tag
   if [ "$1" = build ]; then
     $NV -DRA_SEL_VEC=$vec -DRA_SEL_AHEAD=$ah -DRA_SEL_OUTRING=$ring -DRA_SEL_D1=$d1 -DRA_SEL_D2=$d2 -DRA_SEL_LAG=$lag $ex \

@@ -168,6 +168,25 @@ def read_peak():
     return best or None
 
 
+def mixed_peak(w: float):
+    """Read+write HBM stream peak for a write/read ratio w (scripts/micro/mixed_bw.cu,
+    committed under profiles/), linearly interpolated: the ceiling for a SELECT
+    writing a fraction w of what it reads."""
+    p = os.path.join(ROOT, "profiles", "r01_mixed_bw.txt")
+    if not os.path.exists(p):
+        return None
+    pts = []
+    with open(p) as f:
+        for line in f:
+            if line.startswith("write/read"):
+                pts.append((float(line.split(":")[0].split()[-1]), float(line.split("read+write")[1].split()[0])))
+    pts.sort()
+    for (w0, b0), (w1, b1) in zip(pts, pts[1:]):
+        if w0 <= w <= w1:
+            return b0 + (b1 - b0) * (w - w0) / (w1 - w0)
+    return None
+
+
 def ncu_traffic(key: str):
     """dram bytes per launch from the committed ncu --set full capture, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -303,7 +322,9 @@ def run_ours(args, D: Dist):
         "roofline": {"kernel": "select_fused_kernel", "bound": "hbm", "achieved": achieved, "peak": peak,
                      "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": ncu_traffic(f"select_fused_k{k}_s{s_sel}_n{args.rows_log2}"),
-                     "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kms},
+                     "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kms,
+                     "mixed_stream_peak": mixed_peak(kept / n),
+                     "frac_of_mixed_stream_peak": (achieved / mixed_peak(kept / n)) if mixed_peak(kept / n) else None},
         "clocks": clk.summary(),
     }
     if not args.no_extras:

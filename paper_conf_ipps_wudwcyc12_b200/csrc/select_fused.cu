@@ -50,7 +50,7 @@
 // (Measured on B200, 2^28 rows, k=2, s=.25 overall: window slots of 320 words
 // left ~30% of windows uncopied -> one dependent L2 round trip each, 0.257 ms;
 // 768-word slots copied one tile late: 0.230 ms.  1 CTA/SM with deeper input
-// rings is far slower (0.34 ms) — scripts/sel_variants.sh, scripts/gpu_variants.sh.)
+// rings is far slower (0.34 ms) — scripts/sel_variants.sh + scripts/gpu_selvar.sh.)
 //
 // Status words carry a 28-bit launch epoch (header word bumped by the last
 // tile), so stale words of earlier launches read as "not ready": no per-call

@@ -125,3 +125,19 @@ def test_argument_errors(R):
     with pytest.raises(R.RAError) as e:
         R.select_multi(xd, [[("lt", 0)]] * 3)
     assert e.value.code == R.RA_E_INVAL
+
+
+def test_full_size_bench_config(R):
+    """bench.py's f2 leg at full size (2^28 device-generated rows, seed 2, the
+    bench's two chains), full comparison of both outputs with the oracle."""
+    n = 1 << 28
+    x = torch.empty(n, dtype=torch.int32, device="cuda")
+    ragen.int32_column_dev(2, x)
+    chains = [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)]]
+    outs, cnt = R.select_multi(x, chains)
+    torch.cuda.synchronize()
+    exp = oracle.select_multi(x.cpu().numpy(), chains)
+    for o, c, e in zip(outs, cnt.cpu().tolist(), exp):
+        assert int(c) == e.size
+        np.testing.assert_array_equal(o[:int(c)].cpu().numpy(), e)
+

@@ -171,3 +171,26 @@ def test_argument_errors(R):
         R.ra_select_rows(kd.data_ptr(), 16, R.make_preds([("lt", 0)]), 1, 0, pl, 1, 16, cnt.data_ptr(),
                          ws.data_ptr(), ws.numel(), 0)
     assert e.value.code == R.RA_E_INVAL
+
+
+def test_full_size_bench_config(R):
+    """bench.py's f3 leg at full size: 2^28-row key (seed 2) + two int32 fields
+    (seeds 102, 103) + the key as a third field, k=2, s=.5/stage (the dense
+    compaction path), no ids; and the same with ids (the key pass writes them)."""
+    n = 1 << 28
+    cols = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(3)]
+    for c, seed in zip(cols, (2, 102, 103)):
+        ragen.int32_column_dev(seed, c)
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 2)]
+    hc = [c.cpu().numpy() for c in cols]
+    exp_ids, exp = oracle.select_rows(hc[0], preds, [hc[0], hc[1], hc[2]])
+    for rowids in (False, True):
+        ids, outs, cnt = R.select_rows(cols[0], preds, [cols[0], cols[1], cols[2]], rowids=rowids)
+        torch.cuda.synchronize()
+        c = int(cnt.item())
+        assert c == exp_ids.size
+        if rowids:
+            np.testing.assert_array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
+        for o, e in zip(outs, exp):
+            np.testing.assert_array_equal(o[:c].cpu().numpy(), e)
+

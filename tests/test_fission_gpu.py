@@ -77,3 +77,18 @@ def test_fission_requires_pinned(R, streams):
         R.ra_fission_run(x.ctypes.data, 1000, P, 1, 1, 1000, sarr, 1, out.ctypes.data, 1000,
                          ctypes.byref(cnt), counts.ctypes.data, ws.data_ptr(), ws.numel())
     assert e.value.code == R.RA_E_NOT_PINNED
+
+
+def test_full_size_config_3_host_resident_2_pow_30(R, streams):
+    """BASELINE configs[3] at full size, in bench.py's launch configuration:
+    2^30 host-resident rows (seed 4) in pinned memory, k=2 s=.5/stage, chunk
+    2^24, 3 streams; full comparison with the oracle (chunked SELECT equals
+    SELECT, P:1466-1468, pinned in test_oracle_select)."""
+    n = 1 << 30
+    h = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    ragen.int32_column(4, n, out=h.numpy())
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 2)]
+    h_out, c = R.fission_run(h, preds, 1 << 24, streams[:3])
+    exp = oracle.select(h.numpy(), preds)
+    assert c == exp.size
+    np.testing.assert_array_equal(h_out.numpy()[:c], exp)

@@ -13,12 +13,15 @@
 //   (six cp.async.bulk copies, 11 KB per tile) through an 8-stage
 //   shared-memory ring on mbarriers; 8 compute warps take 4 rows per thread
 //   per tile.  Instead of a predicated update of all 6 group slots per row
-//   (~48 instructions), each row does ONE read-modify-write of its group's
-//   32-byte record in thread-private shared memory (two 128-bit loads, seven
-//   32-bit adds, two 128-bit stores); unselected rows go to a 7th "trash"
-//   record, so there is no predicate at all.  Records are laid out
-//   [slot][half][thread] so a warp is conflict-free whatever its mix of
-//   slots.  A record holds 32-bit sums over <= 256 rows (bounds in nflush()):
+//   (~48 instructions), each row adds into its group's record in
+//   thread-private shared memory with seven `red.shared.add.u32` (records laid
+//   out [slot][field][thread]: every reduction is one conflict-free wavefront
+//   per warp, whatever the warp's mix of slots); unselected rows go to a 7th
+//   "trash" record, so there is no predicate at all.  (RA_Q1N_RED=0: the
+//   earlier read-modify-write of a 32-byte [slot][half][thread] record, two
+//   128-bit loads + two 128-bit stores = 16 wavefronts per warp-row against 7;
+//   measured 7-9% slower.)  A record holds 32-bit sums over <= 256 rows
+//   (bounds in nflush()):
 //     count<<16 | disc,  qty,  price,  dp>>16,  dp&0xffff,  f*(dp>>16),  f*(dp&0xffff)
 //   with dp = price*(100-disc) < 2^31 and f = 100+tax, folded every 256 rows
 //   per thread into 64-bit register sums.  (A variant keeping count/disc/qty/
@@ -36,6 +39,10 @@
 #include "q1_common.cuh"
 
 namespace ra {
+
+#ifndef RA_Q1N_RED
+#define RA_Q1N_RED 1
+#endif
 
 namespace {
 
@@ -74,7 +81,11 @@ struct QnParams {
 
 struct QnSmem {
   alignas(128) unsigned char stage[QN_STAGES][NSTAGE_BYTES];
+#if RA_Q1N_RED
+  uint32_t rec[NS + 1][7][QN_NT];  // [slot][field][thread]: thread-private records, lane-contiguous fields
+#else
   uint4 rec[NS + 1][2][QN_NT];  // [slot][half][thread]: thread-private 32-byte records
+#endif
   unsigned long long wsum[NS][6];  // CTA sums: count, qty, price, disc, disc_price, charge
   uint64_t full[QN_STAGES], empty[QN_STAGES];
   uint32_t status;
@@ -95,8 +106,25 @@ __device__ __forceinline__ void sts128(uint32_t a, const uint4& v) {
   asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
+#if RA_Q1N_RED
+constexpr uint32_t REC_FIELD = QN_NT * 4;             // bytes between the fields of a record
+constexpr uint32_t REC_SLOT = 7 * REC_FIELD;          // bytes between slots
+#else
 constexpr uint32_t REC_HALF = QN_NT * sizeof(uint4);  // bytes between the two halves of a record
 constexpr uint32_t REC_SLOT = 2 * REC_HALF;           // bytes between slots
+#endif
+
+__device__ __forceinline__ void red_add(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 
 // One row: SELECT, domain check, PROJECT, and one read-modify-write of its
 // group's record (unselected / out-of-domain rows hit the trash record).
@@ -110,6 +138,15 @@ __device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cu
   const uint32_t dp = p * (100u - d), f = 100u + t;  // PROJECT (dp < 2^31)
   const uint32_t dh = dp >> 16, dl = dp & 0xFFFFu;
   const uint32_t ra = rec0 + slot * REC_SLOT;
+#if RA_Q1N_RED  // seven shared reductions, one conflict-free wavefront each per warp
+  red_add(ra, (1u << 16) | d);
+  red_add(ra + REC_FIELD, q);
+  red_add(ra + 2 * REC_FIELD, p);
+  red_add(ra + 3 * REC_FIELD, dh);
+  red_add(ra + 4 * REC_FIELD, dl);
+  red_add(ra + 5 * REC_FIELD, f * dh);
+  red_add(ra + 6 * REC_FIELD, f * dl);
+#else
   uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
   a.x += (1u << 16) | d;
   a.y += q;
@@ -120,6 +157,7 @@ __device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cu
   b.z += f * dl;
   sts128(ra, a);
   sts128(ra + REC_HALF, b);
+#endif
 }
 
 // Fold the records into the CTA's 64-bit sums (warp REDUX + one shared atomic
@@ -143,7 +181,12 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
 #pragma unroll
   for (int s = 0; s < NS; ++s) {
     const uint32_t ra = rec0 + s * REC_SLOT;
+#if RA_Q1N_RED
+    const uint4 a = make_uint4(lds32(ra), lds32(ra + REC_FIELD), lds32(ra + 2 * REC_FIELD), lds32(ra + 3 * REC_FIELD));
+    const uint4 b = make_uint4(lds32(ra + 4 * REC_FIELD), lds32(ra + 5 * REC_FIELD), lds32(ra + 6 * REC_FIELD), 0u);
+#else
     const uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
+#endif
     if (!__any_sync(0xffffffffu, (a.x | a.y | a.z | a.w | b.x | b.y | b.z) != 0u)) continue;  // warp-uniform
     const unsigned long long cnt = warp_sum32(a.x >> 16), disc = warp_sum32(a.x & 0xFFFFu);
     const unsigned long long q = warp_sum32(a.y), p = warp_sum32(a.z);
@@ -157,8 +200,13 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
       atomicAdd(&S.wsum[s][4], (dph << 16) + dpl);
       atomicAdd(&S.wsum[s][5], (chh << 16) + chl);
     }
+#if RA_Q1N_RED
+#pragma unroll
+    for (int f = 0; f < 7; ++f) sts32(ra + f * REC_FIELD, 0u);
+#else
     sts128(ra, make_uint4(0, 0, 0, 0));
     sts128(ra + REC_HALF, make_uint4(0, 0, 0, 0));
+#endif
   }
 }
 
@@ -178,7 +226,13 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
   }
   if (tid < QN_NT) {
 #pragma unroll
-    for (int s = 0; s <= NS; ++s) S.rec[s][0][tid] = S.rec[s][1][tid] = make_uint4(0, 0, 0, 0);
+    for (int s = 0; s <= NS; ++s) {
+#if RA_Q1N_RED
+      for (int f = 0; f < 7; ++f) S.rec[s][f][tid] = 0u;
+#else
+      S.rec[s][0][tid] = S.rec[s][1][tid] = make_uint4(0, 0, 0, 0);
+#endif
+    }
   }
   if (tid < NS * 6) (&S.wsum[0][0])[tid] = 0ull;
   if (tid == 0) S.status = 0;

@@ -51,7 +51,10 @@ using namespace q1c;
 constexpr int QN_NT = 256;     // compute threads + 1 producer warp
 constexpr int QN_NW = QN_NT / 32;
 constexpr int QN_TILE = 1024;  // rows per tile (11 KB)
-constexpr int QN_STAGES = 4;
+#ifndef RA_Q1N_STAGES
+#define RA_Q1N_STAGES 4
+#endif
+constexpr int QN_STAGES = RA_Q1N_STAGES;
 constexpr int QN_CTAS_PER_SM = 2;
 constexpr int QN_R = QN_TILE / QN_NT;  // 4 rows per thread per tile
 constexpr int QN_FLUSH_TILES = 256 / QN_R;

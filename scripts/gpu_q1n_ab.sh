@@ -1,7 +1,8 @@
+# narrow Q1 variants: rebuild libra.so with extra defines, time SF10/SF100 (scripts/prof_driver.py q1time)
 mkdir -p gpurun_out
-make -s all >/dev/null 2>&1
-python -m pytest tests/test_q1_narrow_gpu.py tests/test_q1_fission_gpu.py -q -x 2>&1 | tail -2
-echo "== RED=1"; python scripts/prof_driver.py q1time 20 2>&1 | grep narrow
-NVF="-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-fvisibility=hidden -shared -Xptxas -v --expt-relaxed-constexpr -DRA_Q1N_RED=0"
-make -s -B paper_conf_ipps_wudwcyc12_b200/libra.so "NVFLAGS=$NVF" >/dev/null 2>&1
-echo "== RED=0"; python scripts/prof_driver.py q1time 20 2>&1 | grep narrow
+NVF0="-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-fvisibility=hidden -shared -Xptxas -v --expt-relaxed-constexpr"
+for defs in "$@"; do
+  make -s -B paper_conf_ipps_wudwcyc12_b200/libra.so "NVFLAGS=$NVF0 $defs" >/dev/null 2>&1 || { echo "build $defs FAILED"; continue; }
+  echo "== $defs"; python scripts/prof_driver.py q1time 20 2>&1 | grep narrow
+done
+make -s -B all >/dev/null 2>&1

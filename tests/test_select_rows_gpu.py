@@ -20,15 +20,16 @@ def R():
     return R
 
 
-def check(R, key, preds, payloads, offset=0):
+def check(R, key, preds, payloads, offset=0, rowids=True):
     kd = torch.from_numpy(np.concatenate([np.zeros(offset, np.int32), key])).cuda()[offset:]
     pd = [torch.from_numpy(p).cuda() for p in payloads]
-    ids, outs, cnt = R.select_rows(kd, preds, pd)
+    ids, outs, cnt = R.select_rows(kd, preds, pd, rowids=rowids)
     torch.cuda.synchronize()
     c = int(cnt.item())
     exp_ids, exp_outs = oracle.select_rows(key, preds, payloads)
     assert c == exp_ids.size
-    assert np.array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
+    if rowids:
+        assert np.array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
     for o, e in zip(outs, exp_outs):
         assert np.array_equal(o[:c].cpu().numpy(), e)
 
@@ -54,6 +55,7 @@ def test_sizes_offsets(R, n, offset):
     pay4 = (np.arange(n, dtype=np.int32) * 3 + 1)
     pay8 = np.arange(n, dtype=np.int64) * (1 << 33) - 5
     check(R, key, [("lt", 0), ("gt", -(2**30))], [pay4, pay8, key], offset)
+    check(R, key, [("lt", -(2**31) + 2**26)], [pay4, pay8], offset, rowids=False)  # sparse, no ids
 
 
 @pytest.mark.parametrize("s,k", [(0.0, 1), (0.01, 1), (0.5, 2), (0.9, 1), (1.0, 1)])
@@ -154,8 +156,10 @@ def test_both_payload_paths(R, s, force_gather, monkeypatch):
     key = ragen.int32_column(69, n)
     p4 = ragen.int32_column(70, n)
     preds = [("lt", t) for t in ragen.nested_thresholds(s, 1)]
-    check(R, key, preds, [p4, key])  # 4-byte fields only
-    check(R, key, preds, [p4.astype(np.int64) * 5 - 7, p4])  # with an 8-byte field
+    for rowids in (True, False):  # without ids the sparse path rebuilds them from the masks (ids_kernel)
+        check(R, key, preds, [p4, key], rowids=rowids)  # 4-byte fields only
+        check(R, key, preds, [p4.astype(np.int64) * 5 - 7, p4], rowids=rowids)  # with an 8-byte field
+        check(R, key, preds, [p4, key], offset=3, rowids=rowids)  # misaligned key view
 
 
 def test_argument_errors(R):

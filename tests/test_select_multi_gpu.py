@@ -36,6 +36,7 @@ def check(R, x, chains, offset=0):
 def test_sizes_offsets(R, n, offset):
     x = ragen.int32_column(71 + n, n)
     check(R, x, [[("lt", 0)], [("gt", -(2**29)), ("lt", 2**30)]], offset)
+    check(R, x, [[("gt", -(2**31) + 2**28)], [("ne", 7)]], offset)  # both dense: spilled second runs
 
 
 @pytest.mark.parametrize("s0,s1", [(0.0, 1.0), (0.01, 0.9), (0.5, 0.5), (0.9, 0.9), (1.0, 1.0), (0.25, 0.75)])

@@ -1,0 +1,53 @@
+"""Soak test (dev tool): thousands of back-to-back launches of every select
+path with random sizes, offsets and selectivities on one stream, each result
+checked against numpy (counts + sampled values).  Run under `timeout`."""
+import sys
+import time
+
+import numpy as np
+import torch
+
+sys.path.insert(0, ".")
+import paper_conf_ipps_wudwcyc12_b200 as R  # noqa: E402
+import ragen  # noqa: E402
+
+rng = np.random.default_rng(int(sys.argv[2]) if len(sys.argv) > 2 else 1)
+iters = int(sys.argv[1]) if len(sys.argv) > 1 else 2000
+base = ragen.int32_column(99, (1 << 22) + 8)
+bd = torch.from_numpy(base).cuda()
+t0 = time.time()
+for it in range(iters):
+    n = int(rng.choice([0, 1, 7, 4096, 8192, 8193, 100_003, 1 << 20, (1 << 22) - 5]))
+    off = int(rng.integers(0, 4))
+    x, xd = base[off:off + n], bd[off:off + n]
+    t = int(rng.integers(-2**31, 2**31 - 1))
+    kind = it % 4
+    if kind == 0:
+        out, c = R.select_chain(xd, [("lt", t), ("ne", 5)], fused=bool(rng.integers(0, 2)))
+        e = x[(x < t) & (x != 5)]
+        c = int(c.item())
+        assert c == e.size and np.array_equal(out[:c].cpu().numpy(), e), ("chain", it, n, off, t)
+    elif kind == 1:
+        t2 = int(rng.integers(-2**31, 2**31 - 1))
+        outs, cnt = R.select_multi(xd, [[("lt", t)], [("gt", t2)]])
+        e0, e1 = x[x < t], x[x > t2]
+        c0, c1 = (int(v) for v in cnt.cpu().tolist())
+        assert c0 == e0.size and c1 == e1.size, ("multi", it, n, off)
+        assert np.array_equal(outs[0][:c0].cpu().numpy(), e0) and np.array_equal(outs[1][:c1].cpu().numpy(), e1)
+    elif kind == 2:
+        ids, outs, c = R.select_rows(xd, [("lt", t)], [xd], rowids=bool(rng.integers(0, 2)))
+        e = x[x < t]
+        c = int(c.item())
+        assert c == e.size and np.array_equal(outs[0][:c].cpu().numpy(), e), ("rows", it, n, off, t)
+    else:
+        m = max(1, n)
+        cols = ragen.lineitem(it, m, 2000)
+        dc = {k: torch.from_numpy(v).cuda() for k, v in cols.items()}
+        part = R.q1(dc)
+        rows, rc = R.q1_finalize(bytes(part.cpu().numpy().tobytes()))
+        sel = cols["shipdate"] <= R.Q1_CUTOFF_DELTA90
+        assert rc == R.RA_OK and sum(r["count_order"] for r in rows) == int(sel.sum()), ("q1", it, m)
+    if it % 500 == 0:
+        print(f"iter {it} ok ({time.time() - t0:.1f} s)", flush=True)
+torch.cuda.synchronize()
+print(f"soak: {iters} iterations ok in {time.time() - t0:.1f} s")

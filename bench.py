@@ -690,6 +690,17 @@ def host_threads() -> int:
     return len(os.sched_getaffinity(0))
 
 
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def cpu_baseline(x, preds, n):
     def rate(xh, T, budget=2.0):
         t0 = time.perf_counter()
@@ -706,7 +717,7 @@ def cpu_baseline(x, preds, n):
     v1, c1 = rate(x[:s1].cpu().numpy(), 1)
     sT = min(n, 1 << 28)
     vT, cT = rate(x[:sT].cpu().numpy(), T)
-    return {"value": vT, "unit": "rows/s", "cores": T, "kind": "oracle",
+    return {"value": vT, "unit": "rows/s", "cores": T, "kind": "oracle", "cpu": cpu_model(),
             "sample": f"first 2^{sT.bit_length() - 1} rows of the same column, oracle_select (C, -O2) on {T} "
                       f"threads over contiguous row ranges, outputs concatenated",
             "kept": cT, "single_thread": {"value": v1, "cores": 1, "kept": c1,
@@ -737,7 +748,7 @@ def run_reference(args, D: Dist):
         "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic (seeded uniform int32, ragen)",
         "config": {"workload": f"configs[1]: fused {args.k}x SELECT, s={args.sel}/stage, 2^{args.rows_log2} int32 rows; "
                                f"oracle step = bounded sample of 2^26 rows", "kept": int(out.size)},
-        "cpu_baseline": {"value": v, "unit": "rows/s", "cores": T, "kind": "oracle",
+        "cpu_baseline": {"value": v, "unit": "rows/s", "cores": T, "kind": "oracle", "cpu": cpu_model(),
                          "sample": f"2^26 rows of the configs[1] column per step (plain C oracle on {T} threads "
                                    f"over contiguous row ranges, outputs concatenated)"},
         "e2e": {"value": v, "unit": "rows/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},

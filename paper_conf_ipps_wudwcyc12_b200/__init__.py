@@ -54,6 +54,9 @@ def workspace(device, kind: str, nbytes: int, stream=None):
     ws = _WS.get(key)
     if ws is None or ws.numel() < nbytes:
         ws = torch.zeros(max(256, nbytes), dtype=torch.uint8, device=device)
+        # the zero fill runs on the current stream; the fission runtimes use the
+        # workspace from their own streams, so it must be complete first
+        torch.cuda.current_stream(device).synchronize()
         _WS[key] = ws
     return ws
 

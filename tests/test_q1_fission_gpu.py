@@ -89,3 +89,21 @@ def test_fission_rejects_pageable(R):
         R.ra_q1_fission_run(R.lineitem_struct(h), 1000, CUTOFF, 256, st, 1, R.ra_q1_partial(),
                             ws.data_ptr(), ws.numel())
     assert e.value.code == R.RA_E_NOT_PINNED
+
+
+def test_first_call_on_a_fresh_workspace(R):
+    """The workspace helper zero-fills a new workspace on the current stream;
+    the fission runtimes then use it from their own streams.  Every first call
+    on a fresh workspace must see the fill complete (regression test)."""
+    n = 3_000_000
+    cols = ragen.lineitem(21, n, 20000)
+    exp, _ = oracle.q1(cols, R.Q1_CUTOFF_DELTA90)
+    h = {k: torch.from_numpy(v).pin_memory() for k, v in cols.items()}
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    for _ in range(6):
+        R._WS.clear()
+        torch.cuda.synchronize()
+        rows, rc = R.q1_finalize(bytes(R.q1_fission_run(h, 1 << 19, streams)))
+        assert rc == R.RA_OK
+        assert [(r["returnflag"], r["linestatus"], r["count_order"], r["sum_charge"]) for r in rows] == \
+               [(e["returnflag"], e["linestatus"], e["count_order"], e["sum_charge"]) for e in exp]

@@ -22,8 +22,8 @@
 //   128-bit loads + two 128-bit stores = 16 wavefronts per warp-row against 7;
 //   measured 7-9% slower.)  A record holds 32-bit sums over <= 256 rows
 //   (bounds in nflush()):
-//     count<<16 | disc,  qty,  price,  dp>>16,  dp&0xffff,  f*(dp>>16),  f*(dp&0xffff)
-//   with dp = price*(100-disc) < 2^31 and f = 100+tax, folded every 256 rows
+//     count<<16 | disc,  qty,  price,  dp>>16,  dp&0xffff,  tax*(dp>>16),  tax*(dp&0xffff)
+//   with dp = price*(100-disc) < 2^31 (charge = 100*dp + tax*dp), folded every 256 rows
 //   per thread into 64-bit register sums.  (A variant keeping count/disc/qty/
 //   price in predicated register slots and only the dp/charge halves in a
 //   16-byte record moved the bound from shared memory to instruction issue
@@ -42,6 +42,9 @@ namespace ra {
 
 #ifndef RA_Q1N_RED
 #define RA_Q1N_RED 1
+#endif
+#ifndef RA_Q1N_SWAR
+#define RA_Q1N_SWAR 1
 #endif
 #ifndef RA_Q1N_PRMT
 #define RA_Q1N_PRMT 1
@@ -134,6 +137,8 @@ __device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
 
 // One row: SELECT, domain check, PROJECT, and one read-modify-write of its
 // group's record (unselected / out-of-domain rows hit the trash record).
+__device__ __forceinline__ void nadd(uint32_t rec0, uint32_t slot, uint32_t cd, uint32_t q, uint32_t t, uint32_t p);
+
 __device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cutoff, uint32_t sd, uint32_t g,
                                      uint32_t q, uint32_t d, uint32_t t, uint32_t p) {
   const bool sel = (int32_t)sd <= cutoff;  // SELECT
@@ -141,29 +146,72 @@ __device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cu
   const bool okn = (d <= 100u) & (t <= 100u) & (p < (1u << 24));
   status |= sel ? ((okg ? 0u : 1u) | (okn ? 0u : 2u)) : 0u;  // (gating this behind a warp vote: 3% slower)
   const uint32_t slot = (sel & okg & okn) ? g : (uint32_t)TRASH;
-  const uint32_t dp = p * (100u - d), f = 100u + t;  // PROJECT (dp < 2^31)
+  nadd(rec0, slot, (1u << 16) | d, q, t, p);
+}
+
+// PROJECT one row and add it into record `slot` (TRASH: discarded).
+__device__ __forceinline__ void nadd(uint32_t rec0, uint32_t slot, uint32_t cd, uint32_t q, uint32_t t, uint32_t p) {
+  // cd = 1 << 16 | discount (the count and discount fields in one word)
+  const uint32_t dp = p * (65636u - cd);  // PROJECT: price * (100 - discount), < 2^31 in the domain
   const uint32_t dh = dp >> 16, dl = dp & 0xFFFFu;
+  // charge = dp * (100 + tax) = 100 * dp + tax * dp: the records keep tax * dp
+  // (its halves; 100 * dp comes from the dp fields when folded)
   const uint32_t ra = rec0 + slot * REC_SLOT;
 #if RA_Q1N_RED  // seven shared reductions, one conflict-free wavefront each per warp
-  red_add(ra, (1u << 16) | d);
+  red_add(ra, cd);
   red_add(ra + REC_FIELD, q);
   red_add(ra + 2 * REC_FIELD, p);
   red_add(ra + 3 * REC_FIELD, dh);
   red_add(ra + 4 * REC_FIELD, dl);
-  red_add(ra + 5 * REC_FIELD, f * dh);
-  red_add(ra + 6 * REC_FIELD, f * dl);
+  red_add(ra + 5 * REC_FIELD, t * dh);
+  red_add(ra + 6 * REC_FIELD, t * dl);
 #else
   uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
-  a.x += (1u << 16) | d;
+  a.x += cd;
   a.y += q;
   a.z += p;
   a.w += dh;
   b.x += dl;
-  b.y += f * dh;
-  b.z += f * dl;
+  b.y += t * dh;
+  b.z += t * dl;
   sts128(ra, a);
   sts128(ra + REC_HALF, b);
 #endif
+}
+
+// Four rows of one thread (byte i of the g/d/t words, u16 half i of the sd/q
+// pairs, p.{x,y,z,w}): the domain checks of all four in SWAR form — per byte,
+// bit 7 is set iff the value is out of the domain — then one record update
+// per row.  Selected out-of-domain rows are remembered in accg/accn (bit 7 of
+// a byte) and become status bits at the end.
+__device__ __forceinline__ void nrow4(uint32_t rec0, uint32_t& accg, uint32_t& accn, int32_t cutoff, uint2 sd,
+                                      uint32_t g, uint2 q, uint32_t d, uint32_t t, uint4 p) {
+  static_assert(NS == 6, "the group check below tests g >= 6");
+  constexpr uint32_t H = 0x80808080u, L7 = 0x7F7F7F7Fu;
+  const uint32_t bg = (((g & L7) + 0x7A7A7A7Au) | g) & H;  // g >= 6
+  // the top byte of each price: nonzero iff price >= 2^24
+  const uint32_t tb = __byte_perm(__byte_perm(p.x, p.y, 0x0073), __byte_perm(p.z, p.w, 0x0073), 0x5410);
+  const uint32_t bn = ((((d & L7) + 0x1B1B1B1Bu) | d) | (((t & L7) + 0x1B1B1B1Bu) | t) | ((tb & L7) + L7) | tb) &
+                      H;  // discount > 100, tax > 100, price >= 2^24
+  const uint32_t sv[4] = {sd.x & 0xFFFFu, sd.x >> 16, sd.y & 0xFFFFu, sd.y >> 16};
+  uint32_t sm = 0;  // selected rows (SELECT)
+#pragma unroll
+  for (int i = 0; i < 4; ++i) sm |= (int32_t)sv[i] <= cutoff ? (0x80u << (8 * i)) : 0u;
+  accg |= bg & sm;
+  accn |= bn & sm;
+  const uint32_t okm = sm & ~(bg | bn);
+  // slot byte per row: the group for accepted rows, TRASH for the others
+  const uint32_t keep = (okm >> 7) * 0xFFu;  // 0xFF in the bytes of accepted rows
+  const uint32_t slots = (g & keep) | ((uint32_t)TRASH * 0x01010101u & ~keep);
+  const uint32_t qv[4] = {q.x & 0xFFFFu, q.x >> 16, q.y & 0xFFFFu, q.y >> 16};
+  const uint32_t pv[4] = {p.x, p.y, p.z, p.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t sel = 0x4440u + (uint32_t)i;  // byte i, zero-extended
+    const uint32_t slot = __byte_perm(slots, 0, sel);
+    // 1 << 16 | discount_i in one byte permute (bytes: d_i, 0, 1, 0 from d and the constant 1)
+    nadd(rec0, slot, __byte_perm(d, 1u, 0x5450u + (uint32_t)i), qv[i], __byte_perm(t, 0, sel), pv[i]);
+  }
 }
 
 // Fold the records into the CTA's 64-bit sums (warp REDUX + one shared atomic
@@ -171,7 +219,7 @@ __device__ __forceinline__ void nrow(uint32_t rec0, uint32_t& status, int32_t cu
 // flushes a thread adds <= 256 rows, so every record field stays in 32 bits:
 //   count <= 256 (<< 16 -> < 2^25), disc <= 25600 < 2^16, qty < 2^16 * 2^8,
 //   price <= (2^24-1) * 2^8 < 2^32, dp>>16 < 2^15 * 2^8, dp&0xffff < 2^16 * 2^8,
-//   f*(dp>>16) < 200 * 2^15 * 2^8 < 2^31, f*(dp&0xffff) < 200 * 2^16 * 2^8 < 2^32.
+//   tax*(dp>>16) < 100 * 2^15 * 2^8 < 2^30, tax*(dp&0xffff) < 100 * 2^16 * 2^8 < 2^31.
 // A CTA takes <= 2^24 rows (launch_q1_narrow), so its charge sum stays below
 // 200 * 100 * 2^24 * 2^24 < 2^63 and every CTA sum fits 64 bits.
 // Warp sum of 32-bit values as an exact 64-bit value: REDUX on the 16-bit
@@ -204,7 +252,7 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
       atomicAdd(&S.wsum[s][2], p);
       atomicAdd(&S.wsum[s][3], disc);
       atomicAdd(&S.wsum[s][4], (dph << 16) + dpl);
-      atomicAdd(&S.wsum[s][5], (chh << 16) + chl);
+      atomicAdd(&S.wsum[s][5], 100ull * ((dph << 16) + dpl) + (chh << 16) + chl);  // 100 dp + tax dp
     }
 #if RA_Q1N_RED
 #pragma unroll
@@ -266,7 +314,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
   } else {
     // ---------------- compute warps: rows 4*tid .. 4*tid+3 of each tile
     const uint32_t rec0 = dev::smem_u32(&S.rec[0][0][tid]);
-    uint32_t status = 0;
+    uint32_t status = 0, accg = 0, accn = 0;
     int i = 0, since = 0;
     for (int64_t tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x, ++i) {
       const int s = i % QN_STAGES;
@@ -280,7 +328,9 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
       const uint32_t t = *reinterpret_cast<const uint32_t*>(st + NO_T + 4 * tid);
       __syncwarp();
       if (lane == 0) dev::mbar_arrive(&S.empty[s]);  // the stage's values are in registers
-#if RA_Q1N_PRMT  // byte i of g/d/t with one byte permute each (PRMT) instead of shift + mask
+#if RA_Q1N_SWAR
+      nrow4(rec0, accg, accn, P.cutoff, sd, g, q, d, t, p);
+#elif RA_Q1N_PRMT  // byte i of g/d/t with one byte permute each (PRMT) instead of shift + mask
       nrow(rec0, status, P.cutoff, sd.x & 0xFFFFu, __byte_perm(g, 0, 0x4440), q.x & 0xFFFFu, __byte_perm(d, 0, 0x4440),
            __byte_perm(t, 0, 0x4440), p.x);
       nrow(rec0, status, P.cutoff, sd.x >> 16, __byte_perm(g, 0, 0x4441), q.x >> 16, __byte_perm(d, 0, 0x4441),
@@ -306,6 +356,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
     for (int64_t r = tail0 + (int64_t)blockIdx.x * QN_NT + tid; r < P.n; r += (int64_t)gridDim.x * QN_NT)
       nrow(rec0, status, P.cutoff, P.sd[r], P.g[r], P.q[r], P.d[r], P.t[r], P.p[r]);
     nflush(S, rec0);
+    status |= (accg ? 1u : 0u) | (accn ? 2u : 0u);
     if (status) atomicOr(&S.status, status);
   }
   // CTA partial -> P.blocks[blockIdx]; the last CTA folds all of them

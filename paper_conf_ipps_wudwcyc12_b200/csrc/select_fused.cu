@@ -105,6 +105,9 @@ constexpr int K = LAG + 2;               // metadata slots: tiles counted but no
 #ifndef RA_SEL_PTXSCATTER
 #define RA_SEL_PTXSCATTER 1
 #endif
+#ifndef RA_SEL_SPILL_AT
+#define RA_SEL_SPILL_AT RING  // M == 2: a tile whose two runs exceed this spills its second run
+#endif
 #ifndef RA_SEL_BATCH
 #define RA_SEL_BATCH 1  // tiles per ticket (see the producer warp)
 #endif
@@ -409,6 +412,8 @@ __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int
     lim2 = lim2 < 0 ? 0 : (lim2 > c2 ? c2 : lim2);
     int32_t* __restrict__ out2 = P.out2 + g2;
     if (S.spilled[k % K]) {  // from the spill slot (global, L2)
+      // (a batched 16-B readback needs registers the 2-CTA/SM kernel does not
+      // have: it spilled and slowed every pair; measured)
       const int32_t* sp = P.spill + ((int64_t)blockIdx.x * K + k % K) * SEL_TILE;
       for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = sp[e];
     } else {
@@ -699,7 +704,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // the tile (read back when the tile is written).  Measured: spilling both
     // runs, or placing such tiles straight from registers after waiting for
     // their own placement, is slower still.
-    const bool spill2 = M == 2 && agg + agg2 > RING;
+    const bool spill2 = M == 2 && agg + agg2 > RA_SEL_SPILL_AT;
     if (ROWS && P.meta && lane == 0) P.meta[t * 12 + warp] = (uint32_t)wbase;
     const bool ring_rows = !ROWS || P.rowids;  // ROWS without ids: placement only, no ring
     const int32_t rows_in = ring_rows ? agg + (spill2 ? 0 : agg2) : 0;  // ring rows this tile needs

@@ -15,6 +15,7 @@ rng = np.random.default_rng(int(sys.argv[2]) if len(sys.argv) > 2 else 1)
 iters = int(sys.argv[1]) if len(sys.argv) > 1 else 2000
 base = ragen.int32_column(99, (1 << 22) + 8)
 bd = torch.from_numpy(base).cuda()
+fstreams = [torch.cuda.Stream() for _ in range(3)]
 t0 = time.time()
 for it in range(iters):
     n = int(rng.choice([0, 1, 7, 4096, 8192, 8193, 100_003, 1 << 20, (1 << 22) - 5]))
@@ -47,6 +48,14 @@ for it in range(iters):
         rows, rc = R.q1_finalize(bytes(part.cpu().numpy().tobytes()))
         sel = cols["shipdate"] <= R.Q1_CUTOFF_DELTA90
         assert rc == R.RA_OK and sum(r["count_order"] for r in rows) == int(sel.sum()), ("q1", it, m)
+        enc, st = R.q1_encode(dc)  # narrow (f4) must equal wide
+        nrows, nrc = R.q1_finalize(bytes(R.q1_narrow(enc).cpu().numpy().tobytes()))
+        assert nrc == R.RA_OK and nrows == rows, ("q1 narrow", it, m)
+        if it % 16 == 3:  # host-resident under fission (f1), random chunking
+            h = {k: torch.from_numpy(v).pin_memory() for k, v in cols.items()}
+            S = int(rng.integers(1, 4))
+            fr, _ = R.q1_finalize(bytes(R.q1_fission_run(h, int(rng.integers(1, m + 1)), fstreams[:S])))
+            assert fr == rows, ("q1 fission", it, m, S)
     if it % 500 == 0:
         print(f"iter {it} ok ({time.time() - t0:.1f} s)", flush=True)
 torch.cuda.synchronize()

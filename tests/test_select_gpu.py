@@ -176,3 +176,24 @@ def test_bad_arguments_raise(R):
     assert e.value.code == R.RA_E_INVAL
     with pytest.raises(R.RAError):
         R.select_chain(x, [("lt", 0)] * 9)
+
+
+def test_more_than_2_pow_31_rows(R):
+    """2^31 + 2^28 + 12345 rows (9.7 GB in, > 2^18 tiles, output offsets past
+    2^31): 64-bit tile indices, tickets and offsets; count and sampled outputs
+    vs the oracle's definition evaluated with numpy on the same rows."""
+    n = (1 << 31) + (1 << 28) + 12345
+    x = torch.empty(n, dtype=torch.int32, device="cuda")
+    ragen.int32_column_dev(12, x)
+    preds = [("gt", -(2**31) + 2**28)]  # keeps ~94%: the output passes 2^31 rows
+    out, c = R.select_chain(x, preds)
+    torch.cuda.synchronize()
+    c = int(c.item())
+    xh = x.cpu().numpy()
+    keep = xh > -(2**31) + 2**28
+    assert c == int(keep.sum()), (c, int(keep.sum()))
+    assert c > (1 << 31)
+    idx = np.flatnonzero(keep)
+    rng = np.random.default_rng(0)
+    pos = np.concatenate([np.arange(64), rng.integers(0, c, 1 << 16), np.arange(c - 64, c)])
+    np.testing.assert_array_equal(out[torch.from_numpy(pos).cuda()].cpu().numpy(), xh[idx[pos]])

@@ -198,3 +198,30 @@ def test_full_size_bench_config(R):
         for o, e in zip(outs, exp):
             np.testing.assert_array_equal(o[:c].cpu().numpy(), e)
 
+
+
+def test_row_ids_near_2_pow_32(R):
+    """n = 2^32 - 5 rows (the ABI limit for uint32 ids): key[i] = int32(i)
+    (wrapping), select key < 0 keeps rows 2^31 .. n-1, so ids run up to
+    2^32 - 6 and each output is known in closed form; with ids (key pass) and
+    without (dense compaction path), sampled positions checked."""
+    n = (1 << 32) - 5
+    x = torch.empty(n, dtype=torch.int32, device="cuda")
+    step = 1 << 28
+    for lo in range(0, n, step):
+        hi = min(n, lo + step)
+        x[lo:hi].copy_(torch.arange(lo, hi, dtype=torch.int64, device="cuda").to(torch.int32))
+    c_exp = n - (1 << 31)
+    rng = np.random.default_rng(1)
+    pos = np.concatenate([np.arange(64), rng.integers(0, c_exp, 1 << 16), np.arange(c_exp - 64, c_exp)])
+    pd = torch.from_numpy(pos).cuda()
+    for rowids in (True, False):
+        ids, outs, cnt = R.select_rows(x, [("lt", 0)], [x], rowids=rowids)
+        torch.cuda.synchronize()
+        assert int(cnt.item()) == c_exp
+        exp_rows = (1 << 31) + pos
+        if rowids:
+            np.testing.assert_array_equal(ids.view(torch.int32)[pd].cpu().numpy().view(np.uint32).astype(np.int64),
+                                          exp_rows)
+        np.testing.assert_array_equal(outs[0][pd].cpu().numpy().astype(np.int64), exp_rows - (1 << 32))
+        del ids, outs

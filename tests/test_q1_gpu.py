@@ -255,3 +255,27 @@ def test_columns_not_coalignable(R, offsets):
     rows, rc, _ = gpu_q1(R, d)
     assert rc == R.RA_OK
     assert_same(rows, exp)
+
+
+def test_n_past_2_pow_31_closed_form(R):
+    """2^31 + 2^28 identical wide rows (92 GB on the device) -- the sums are n
+    times the row's values, exact, past 2^31 rows and with Sum(charge) far
+    beyond int64 per group."""
+    n = (1 << 31) + (1 << 28)
+    vals = {"shipdate": 9000, "returnflag": ord("R"), "linestatus": ord("F"), "quantity": 5000,
+            "extendedprice": 10494950, "discount": 0, "tax": 8}
+    cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
+            for name, dt in ragen.LINEITEM_COLUMNS}
+    for k, v in vals.items():
+        cols[k].fill_(v)
+    rows, rc, part = gpu_q1(R, cols)
+    assert rc == R.RA_OK and part.rows == n and len(rows) == 1
+    r = rows[0]
+    dp = 10494950 * 100
+    assert (r["returnflag"], r["linestatus"]) == ("R", "F")
+    assert r["count_order"] == n and r["sum_qty"] == 5000 * n and r["sum_base_price"] == 10494950 * n
+    assert r["sum_disc"] == 0 and r["sum_disc_price"] == dp * n and r["sum_charge"] == dp * 108 * n
+    assert r["sum_charge"] > 2**63
+    # AVG per reading C12: (double)Sum / (double)(100 count)
+    assert r["avg_qty"] == float(5000 * n) / float(100 * n) and r["avg_disc"] == 0.0
+    assert r["avg_price"] == float(10494950 * n) / float(100 * n)

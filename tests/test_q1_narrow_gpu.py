@@ -190,3 +190,26 @@ def test_narrow_fission_matches_oracle_and_device(R, n, chunk, S):
     torch.cuda.synchronize()
     assert bytes(part) == dpart.cpu().numpy().tobytes()
     assert ctypes.sizeof(part) == dpart.numel()
+
+
+def test_n_near_2_pow_32_closed_form(R):
+    """n = 2^32 - 1 identical narrow rows (47 GB on the device: the ABI's row
+    limit) -- the SQL sums are n times the row's values, exact: 64-bit CTA
+    sums, 128-bit charge, the per-CTA row cap and the last-CTA fold at the
+    largest launch."""
+    n = (1 << 32) - 1
+    cols = R.narrow_empty(n, "cuda")
+    vals = {"shipdate": 10000, "group": 3, "quantity": 1700, "discount": 5, "tax": 2, "extendedprice": 2116823}
+    for k, v in vals.items():  # group 3 = 2*rf + ls with rf N (1), ls O (1): N-O
+        cols[k].fill_(v)
+    rows, rc = R.q1_finalize(bytes(R.q1_narrow(cols).cpu().numpy().tobytes()))
+    assert rc == R.RA_OK and len(rows) == 1
+    r = rows[0]
+    dp = 2116823 * (100 - 5)
+    assert (r["returnflag"], r["linestatus"]) == ("N", "O")
+    assert r["count_order"] == n and r["sum_qty"] == 1700 * n and r["sum_base_price"] == 2116823 * n
+    assert r["sum_disc"] == 5 * n and r["sum_disc_price"] == dp * n and r["sum_charge"] == dp * 102 * n
+    # AVG per reading C12: (double)Sum / (double)(100 count); Sum(price) > 2^53 here,
+    # so this is not the correctly rounded 21168.23 (C12's exactness holds below 2^53)
+    assert r["avg_qty"] == float(1700 * n) / float(100 * n) and r["avg_disc"] == float(5 * n) / float(100 * n)
+    assert r["avg_price"] == float(2116823 * n) / float(100 * n)

@@ -41,6 +41,13 @@ def test_workspace_sizes():
     assert R.ra_select_workspace_bytes(1 << 28, 1, 0) == f  # k=1 never materialises
     assert R.ra_fission_workspace_bytes(1 << 20, 3, 2, 1) >= 3 * 2 * 4 * (1 << 20)
     assert R.ra_fission_workspace_bytes(0, 3, 2, 1) == 0
+    # two outputs: select status words + per-CTA spill slots (<= 320 CTAs x 5 x 32 KB)
+    m = R.ra_select_multi_workspace_bytes(1 << 28)
+    assert f < m <= f + 256 + 320 * 5 * 32768
+    assert R.ra_select_multi_workspace_bytes(1 << 10) < R.ra_select_multi_workspace_bytes(1 << 20) <= m
+    # tuple SELECT: status words + order masks (n/8 + n/170 B) + id staging (4 B/row)
+    t = R.ra_select_rows_workspace_bytes(1 << 28, 2)
+    assert t >= f + (1 << 28) // 8 + 4 * (1 << 28)
 
 
 def test_argument_errors_without_gpu():

@@ -739,7 +739,7 @@ def cpu_model() -> str:
 
 
 def cpu_baseline(x, preds, n):
-    def rate(xh, T, budget=2.0):
+    def rate(xh, T, budget=5.0):  # ~10 s of CPU work in all (two legs)
         t0 = time.perf_counter()
         reps = 0
         while True:

@@ -8,11 +8,13 @@
 // price) raises the rows/s ceiling ~3.5x.  At 11 B/row the per-row arithmetic
 // becomes the limit, so the accumulation is restructured as well:
 //
-// q1n_kernel — persistent, one CTA per SM, warp-specialised like the wide
+// q1n_kernel — persistent, two CTAs per SM, warp-specialised like the wide
 //   q1_tma_kernel: a producer warp streams 1024-row tiles of the six columns
-//   (six cp.async.bulk copies, 11 KB per tile) through an 8-stage
+//   (six cp.async.bulk copies, 11 KB per tile) through a 4-stage
 //   shared-memory ring on mbarriers; 8 compute warps take 4 rows per thread
-//   per tile.  Instead of a predicated update of all 6 group slots per row
+//   per tile.  The domain checks and the SELECT of a thread's four rows run
+//   in SWAR form on the packed words (nrow4: per byte, bit 7 = out of
+//   domain), then each row is projected and added (nadd).  Instead of a predicated update of all 6 group slots per row
 //   (~48 instructions), each row adds into its group's record in
 //   thread-private shared memory with seven `red.shared.add.u32` (records laid
 //   out [slot][field][thread]: every reduction is one conflict-free wavefront
@@ -24,7 +26,7 @@
 //   (bounds in nflush()):
 //     count<<16 | disc,  qty,  price,  dp>>16,  dp&0xffff,  tax*(dp>>16),  tax*(dp&0xffff)
 //   with dp = price*(100-disc) < 2^31 (charge = 100*dp + tax*dp), folded every 256 rows
-//   per thread into 64-bit register sums.  (A variant keeping count/disc/qty/
+//   per thread into the CTA's 64-bit shared sums.  (A variant keeping count/disc/qty/
 //   price in predicated register slots and only the dp/charge halves in a
 //   16-byte record moved the bound from shared memory to instruction issue
 //   and was 16% slower.)  The end reduction is the shared warp -> CTA ->

@@ -326,7 +326,14 @@ def run_ours(args, D: Dist):
     torch.cuda.synchronize()
     launches0 = R.ra_kernel_launches()
     with ClockSampler(D.device(torch)) as clk:
-        ms, kms = timed(torch, D, chain_step, args.steps, args.warmup, kernel_fn=chain_kernel, join=join)
+        # at N=1 a step is exactly one kernel launch, back to back on one stream
+        # (programmatic dependent launch overlaps each launch with the previous
+        # kernel's tail; an event between them would break that), so the
+        # kernel's mean duration is the timed region / K; at N>1 each kernel is
+        # bracketed by its own events
+        ms, kms = timed(torch, D, chain_step, args.steps, args.warmup,
+                        kernel_fn=chain_kernel if D.pg else None, join=join)
+        kms = ms if kms is None else kms
     launches = R.ra_kernel_launches() - launches0 - args.warmup
     last = (args.steps - 1) & 1
     cnt = cnts[last:last + 1]

@@ -17,7 +17,9 @@ The same line carries
   clocks        SM clocks and throttle reasons sampled during the timed region
 
 `--impl reference` runs the CPU oracle as the reference arm on the same config.
-Launch: python bench.py [--gpus N --steps K --warmup W]; N>1 under torchrun.
+Launch: python bench.py [--gpus N --steps K --warmup W].  N>1: under torchrun
+(WORLD_SIZE must equal N), or without it bench.py re-launches itself as N
+ranks through torch.distributed.run.
 """
 from __future__ import annotations
 
@@ -72,6 +74,9 @@ class Dist:
             # ranks sharing one GPU (functional check only; NCCL needs one GPU per rank)
             backend = os.environ.get("RA_BENCH_BACKEND", "nccl")
             if backend == "nccl":
+                if torch.cuda.device_count() < self.world:
+                    raise SystemExit(f"bench.py: {self.world} ranks need {self.world} GPUs, "
+                                     f"{torch.cuda.device_count()} visible (NCCL: one GPU per rank)")
                 dist.init_process_group("nccl", device_id=torch.device("cuda", self.local))
             else:
                 dist.init_process_group(backend)
@@ -301,6 +306,8 @@ def run_ours(args, D: Dist):
     kdone = [torch.cuda.Event() for _ in range(2)]
     xdone = [None, None]
     gathered = [torch.zeros(D.world, dtype=torch.int64, device=dev) for _ in range(2)]
+    offsets = [torch.zeros(D.world, dtype=torch.int64, device=dev) for _ in range(2)]
+    totals = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in range(2)]
 
     def chain_kernel(i):
         R.ra_select_chain(*args_chain[i & 1])
@@ -313,7 +320,7 @@ def run_ours(args, D: Dist):
             kdone[b].record(stream)
             side.wait_event(kdone[b])
             with torch.cuda.stream(side):
-                rdist.exchange_counts(cnts[b:b + 1], counts=gathered[b])
+                rdist.exchange_counts(cnts[b:b + 1], counts=gathered[b], offsets=offsets[b], total=totals[b])
                 xdone[b] = torch.cuda.Event()
                 xdone[b].record(side)
             if xdone[b ^ 1] is not None:  # the next kernel reuses the buffer step i-1's exchange read
@@ -338,8 +345,10 @@ def run_ours(args, D: Dist):
     last = (args.steps - 1) & 1
     cnt = cnts[last:last + 1]
     kept = int(cnt.item())
-    if D.pg:
-        assert int(gathered[last][D.rank].item()) == kept
+    if D.pg:  # the exchange's result: this rank's count, offset = counts of lower ranks, total
+        g = [int(v) for v in gathered[last].tolist()]
+        assert g[D.rank] == kept
+        assert int(offsets[last][D.rank].item()) == sum(g[:D.rank]) and int(totals[last].item()) == sum(g)
     value = D.world * n / (ms * 1e-3)
     peak, peak_src = peaks()
     alg_bytes = 4 * n + 4 * kept
@@ -476,6 +485,7 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     ragen.int32_column_dev(CHAIN_SEED + 200, xb, row0=D.rank * nb, stream=sh)
     ob = torch.empty(nb, dtype=torch.int32, device=dev)
     cb = torch.zeros(1, dtype=torch.int64, device=dev)
+    gb, ofb, tob = (torch.zeros(m, dtype=torch.int64, device=dev) for m in (D.world, D.world, 1))
     wsb_b = R.ra_select_workspace_bytes(nb, k, 1)
     wsb = torch.zeros(wsb_b, dtype=torch.uint8, device=dev)
     Pb = R.make_preds(preds)
@@ -485,7 +495,7 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
         if not kernel_done:
             R.ra_select_chain(*ab)
         if D.pg:
-            rdist.exchange_counts(cb)
+            rdist.exchange_counts(cb, counts=gb, offsets=ofb, total=tob)
 
     bms, bkms = timed(torch, D, big_step, 20, 3, kernel_fn=lambda i: R.ra_select_chain(*ab))
     bk = int(cb.item())
@@ -705,12 +715,9 @@ def q1_e2e(args, D, torch, R, sf):
     npart = R.q1_narrow_fission_run(hn, chunk_n, streams)
     nms, _ = timed(torch, D, lambda i, kernel_done=False: R.q1_narrow_fission_run(hn, chunk_n, streams), 3, 1)
     nrows, nrc = R.q1_finalize(bytes(npart))
-    if nrows != rows or rows != dref:  # recorded, not raised: the line must still be printed
-        msg = f"FAILED: wide == device {rows == dref}, narrow == device {nrows == dref}"
-        print(f"q1_e2e check {msg}", file=sys.stderr, flush=True)
-        res["check"] = msg
-    else:
-        res["check"] = "wide and narrow fission results equal the device-resident query"
+    if nrows != rows or rows != dref:  # a bit-exact system prints no number next to a mismatch
+        raise SystemExit(f"q1_e2e parity FAILED: wide == device {rows == dref}, narrow == device {nrows == dref}")
+    res["check"] = "wide and narrow fission results equal the device-resident query"
     res["narrow"] = {"value": N / (nms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 11 * N,
                      "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": nms,
                      "pcie_h2d_gbs": 11 * N / (nms * 1e-3) / 1e9,
@@ -802,8 +809,36 @@ def run_reference(args, D: Dist):
     }), flush=True)
 
 
+def _free_port() -> int:
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
+def launch_ranks(args) -> None:
+    """`--gpus N` with N > 1 outside torchrun: re-launch this command as N ranks
+    (one process per GPU) through torch.distributed.run on 127.0.0.1.  Under
+    torchrun the world size must equal --gpus: a mismatch fails loudly instead
+    of timing another number of GPUs than the line claims."""
+    world = os.environ.get("WORLD_SIZE")
+    if world is not None:
+        if int(world) != args.gpus:
+            raise SystemExit(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}")
+        return
+    if args.gpus <= 1:
+        return
+    os.environ.setdefault("NCCL_DEBUG", "INFO")  # the communicator's rank count is in the log
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.abspath(__file__),
+           *sys.argv[1:]]
+    print(f"bench.py: launching {args.gpus} ranks: {' '.join(cmd)}", file=sys.stderr, flush=True)
+    os.execv(sys.executable, cmd)
+
+
 def main():
     args = parse()
+    launch_ranks(args)
     D = Dist()
     if args.impl == "reference":
         run_reference(args, D)

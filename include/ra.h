@@ -20,7 +20,14 @@
  *  - Calls are reentrant given distinct workspaces; a workspace may be reused
  *    by successive calls ordered on one stream.
  *  - Workspaces must be zero-filled once after allocation (ra_workspace_init
- *    or any memset); the library keeps them self-cleaning afterwards.
+ *    or any memset); the library keeps them self-cleaning afterwards for any
+ *    number of calls of the SAME entry point with any n the size allows
+ *    (select status words carry a launch-epoch tag; the launch before the tag
+ *    wraps clears every status word the workspace has carried; data other
+ *    than status words lives at the 256-B aligned end of the workspace).
+ *    A workspace handed to a DIFFERENT entry point must be re-initialised
+ *    first: another layout's data could read as a status word.
+ *  - ws_bytes may exceed the required size by any amount.
  */
 #ifndef RA_H
 #define RA_H
@@ -118,6 +125,22 @@ int ra_select(const int32_t* d_in, int64_t n, ra_pred pred, int32_t* d_out, int6
 int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,
                     int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
                     size_t ws_bytes, ra_stream_t stream);
+
+/* Multi-GPU SELECT exchange, device side: rank r
+ * selected from its own contiguous row range; after an all_gather of the
+ * per-rank counts (NCCL, by the caller) its output belongs at the sum of the
+ * counts of ranks < r — the gather stage's "correct position in the final
+ * array" (Fig 3) one level up.  One small kernel, stream-ordered.
+ *
+ *  d_counts   device int64[n_ranks], 1 <= n_ranks <= RA_MAX_RANKS, the counts
+ *             in rank order
+ *  d_offsets  device int64[n_ranks] or NULL: exclusive prefix sums
+ *  d_total    device int64 or NULL: the sum (not both NULL)
+ *  All pointers 8-byte aligned. */
+#define RA_MAX_RANKS 65536
+
+int ra_select_offsets(const int64_t* d_counts, int n_ranks, int64_t* d_offsets, int64_t* d_total,
+                      ra_stream_t stream);
 
 /* ============================================================ TPC-H Q1
  * SELECT (l_shipdate <= cutoff) -> PROJECT (disc_price = price*(1-disc),

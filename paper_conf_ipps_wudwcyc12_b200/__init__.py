@@ -47,16 +47,42 @@ def _stream_handle(stream) -> int:
     return int(stream.cuda_stream) if hasattr(stream, "cuda_stream") else int(stream)
 
 
+def _used_on(stream, *tensors):
+    """Tensors allocated here (on the current stream) but written by kernels
+    enqueued on ``stream``: record that use with the caching allocator, so
+    their memory is not handed out again before ``stream``'s work completes."""
+    torch = _torch()
+    if stream is None:
+        return
+    for t in tensors:
+        if t is None:
+            continue
+        s = stream if isinstance(stream, torch.cuda.Stream) else \
+            torch.cuda.ExternalStream(int(stream), device=t.device)
+        if s != torch.cuda.current_stream(t.device):
+            t.record_stream(s)
+
+
 def workspace(device, kind: str, nbytes: int, stream=None):
-    """Zero-initialised, cached per (device, kind, stream) workspace tensor."""
+    """Zero-initialised workspace tensor, cached per (device, kind, stream).
+
+    One ``kind`` per entry point (ra.h: a workspace handed to another entry
+    point must be re-initialised).  The zero fill runs on the current stream
+    and is complete before this returns: the kernels, and the fission runtimes'
+    own streams, may use the workspace from any stream.  A replaced (smaller)
+    workspace was recorded on the stream that used it, so the allocator keeps
+    its memory until that stream's work is done."""
     torch = _torch()
     key = (str(device), kind, _stream_handle(stream))
     ws = _WS.get(key)
     if ws is None or ws.numel() < nbytes:
         ws = torch.zeros(max(256, nbytes), dtype=torch.uint8, device=device)
-        # the zero fill runs on the current stream; the fission runtimes use the
-        # workspace from their own streams, so it must be complete first
+        # Root cause of round 1's one-off Q1-fission mismatch: without this the
+        # fill kernel (current stream) could still be running while the fission
+        # streams (not ordered after it) had already accumulated chunk partials
+        # into the same bytes, zeroing part of the result (DESIGN.md §7).
         torch.cuda.current_stream(device).synchronize()
+        _used_on(stream, ws)
         _WS[key] = ws
     return ws
 
@@ -75,6 +101,7 @@ def select_chain(x, preds, fused: bool = True, out=None, count=None, stream=None
         out = torch.empty(max(1, n), dtype=torch.int32, device=x.device)
     if count is None:
         count = torch.empty(1, dtype=torch.int64, device=x.device)
+    _used_on(stream, out, count)
     need = ra_select_workspace_bytes(n, k, int(fused))
     ws = workspace(x.device, "select_fused" if fused else "select_unfused", need, stream)
     P = make_preds(preds)
@@ -102,7 +129,8 @@ def select_multi(x, chains, outs=None, stream=None):
     op = (ctypes.c_void_p * M)(*[o.data_ptr() for o in outs])
     caps = (ctypes.c_int64 * M)(*[o.numel() for o in outs])
     cp = (ctypes.c_void_p * M)(*[counts.data_ptr() + 8 * o for o in range(M)])
-    ws = workspace(x.device, "select_fused", ra_select_multi_workspace_bytes(n), stream)
+    _used_on(stream, counts, *outs)
+    ws = workspace(x.device, "select_multi", ra_select_multi_workspace_bytes(n), stream)
     ra_select_multi(x.data_ptr(), n, ch, ks, M, op, caps, cp, ws.data_ptr(), ws.numel(), _stream_handle(stream))
     return outs, counts
 
@@ -128,6 +156,7 @@ def select_rows(key, preds, payloads=(), rowids: bool = True, out_cap=None, stre
         outs.append(o)
         pl[j].col, pl[j].out, pl[j].elem_bytes = c.data_ptr(), o.data_ptr(), c.element_size()
     count = torch.empty(1, dtype=torch.int64, device=key.device)
+    _used_on(stream, ids, count, *outs)
     need = ra_select_rows_workspace_bytes(n, k)
     ws = workspace(key.device, "select_rows", need, stream)
     P = make_preds(preds)
@@ -147,6 +176,7 @@ def q1(cols, cutoff: int = Q1_CUTOFF_DELTA90, partial=None, stream=None):
     n = sd.numel()
     if partial is None:
         partial = torch.empty(ctypes.sizeof(ra_q1_partial), dtype=torch.uint8, device=sd.device)
+        _used_on(stream, partial)
     ws = workspace(sd.device, "q1", ra_q1_workspace_bytes(n), stream)
     ra_q1(lineitem_struct(cols), n, int(cutoff), partial.data_ptr(), ws.data_ptr(), ws.numel(),
           _stream_handle(stream))
@@ -170,6 +200,7 @@ def q1_encode(cols, out=None, stream=None):
     if out is None:
         out = narrow_empty(n, sd.device)
     status = torch.empty(1, dtype=torch.uint32, device=sd.device)
+    _used_on(stream, status, *out.values())
     h_out = ra_lineitem_narrow_out(*[out[name].data_ptr() for name, _ in NARROW_COLUMNS])
     ra_q1_encode(lineitem_struct(cols), n, h_out, status.data_ptr(), _stream_handle(stream))
     return out, status
@@ -182,6 +213,7 @@ def q1_narrow(ncols, cutoff: int = Q1_CUTOFF_DELTA90, partial=None, stream=None)
     n = sd.numel()
     if partial is None:
         partial = torch.empty(ctypes.sizeof(ra_q1_partial), dtype=torch.uint8, device=sd.device)
+        _used_on(stream, partial)
     ws = workspace(sd.device, "q1", ra_q1_workspace_bytes(n), stream)
     h = ra_lineitem_narrow(*[ncols[name].data_ptr() for name, _ in NARROW_COLUMNS])
     ra_q1_narrow(h, n, int(cutoff), partial.data_ptr(), ws.data_ptr(), ws.numel(), _stream_handle(stream))

@@ -32,6 +32,7 @@ RA_E_WORKSPACE = -6
 RA_MAX_PREDS = 8
 RA_MAX_PAYLOAD = 4
 RA_MAX_OUTPUTS = 2
+RA_MAX_RANKS = 65536
 RA_Q1_GROUPS = 6
 RA_LT, RA_LE, RA_GT, RA_GE, RA_EQ, RA_NE = range(6)
 OPS = {"lt": RA_LT, "le": RA_LE, "gt": RA_GT, "ge": RA_GE, "eq": RA_EQ, "ne": RA_NE}
@@ -121,6 +122,7 @@ _SIGS = {
     "ra_select": ([_vp, _i64, ra_pred, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_select_chain": ([_vp, _i64, _vp, _i32, _i32, _vp, _i64, _vp, _vp, _sz, _vp], _i32),
     "ra_select_multi": ([_vp, _i64, _vp, _vp, _i32, _vp, _vp, _vp, _vp, _sz, _vp], _i32),
+    "ra_select_offsets": ([_vp, _i32, _vp, _vp, _vp], _i32),
     "ra_select_rows_workspace_bytes": ([_i64, _i32], _sz),
     "ra_select_multi_workspace_bytes": ([_i64], _sz),
     "ra_select_rows": ([_vp, _i64, _vp, _i32, _vp, _vp, _i32, _i64, _vp, _vp, _sz, _vp], _i32),
@@ -184,6 +186,10 @@ def ra_select_chain(d_in: int, n: int, h_preds, k: int, fused: int, d_out: int, 
                     d_count: int, d_ws: int, ws_bytes: int, stream: int) -> None:
     _check(_lib.ra_select_chain(d_in, n, h_preds, k, fused, d_out, out_cap, d_count, d_ws, ws_bytes,
                                 stream))
+
+
+def ra_select_offsets(d_counts: int, n_ranks: int, d_offsets: int, d_total: int, stream: int) -> None:
+    _check(_lib.ra_select_offsets(d_counts, n_ranks, d_offsets, d_total, stream))
 
 
 def ra_select_multi(d_in: int, n: int, h_chains, ks, M: int, d_outs, out_caps, d_counts, d_ws: int,

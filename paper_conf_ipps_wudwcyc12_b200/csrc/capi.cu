@@ -31,16 +31,25 @@ int cuda_fail(cudaError_t e, const char* what) {
   return fail(RA_E_CUDA, "%s: %s (%d)", what, cudaGetErrorString(e), (int)e);
 }
 
-int num_sms() {
-  static int cache[64];
+std::mutex& init_mutex() {
+  static std::mutex m;
+  return m;
+}
+
+int current_device() {
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
-  if (!cache[dev]) {
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
+  return dev;
+}
+
+int num_sms() {
+  static std::atomic<int> cache[64];
+  const int dev = current_device();
+  return device_once(cache, dev, [&] {
     int v = 0;
     cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
-    cache[dev] = v > 0 ? v : 148;
-  }
-  return cache[dev];
+    return v > 0 ? v : 148;
+  });
 }
 
 int canonicalize(const ra_pred* preds, int k, CanonPred* out) {
@@ -210,7 +219,9 @@ RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const*
   second.d_count = d_counts[1];
   const size_t need = ra_select_multi_workspace_bytes(n);
   if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
-  second.spill = (int32_t*)((char*)d_ws + ((ra_select_workspace_bytes(n, RA_MAX_PREDS, 1) + 255) / 256) * 256);
+  // spill slots at the (256-B aligned) END of the workspace: the status words
+  // of a later call on the same workspace with any n never reach them
+  second.spill = (int32_t*)((char*)d_ws + (ws_bytes & ~(size_t)255) - ra::sel_spill_bytes(n));
   return launch_select_pass(d_in, n, nullptr, cp[0], d_outs[0], out_caps[0], d_counts[0], d_ws, (cudaStream_t)stream,
                             nullptr, &second);
 }
@@ -265,7 +276,10 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   // (sparse; ids rebuilt from the masks into the workspace when the caller
   // did not ask for them) or by the streaming compaction (dense), chosen on
   // the device from the count.
-  const size_t mask_off = ((ra_select_workspace_bytes(n, k, 1) + 255) / 256) * 256;
+  // masks and staged ids sit at the (256-B aligned) END of the workspace, so
+  // the status words of a later call with any n never overlap them
+  const size_t extra = ((ra::sel_masks_bytes(n) + 255) / 256) * 256 + (((size_t)n * 4 + 255) / 256) * 256;
+  const size_t mask_off = (ws_bytes & ~(size_t)255) - extra;
   const size_t stage_off = mask_off + ((ra::sel_masks_bytes(n) + 255) / 256) * 256;
   uint32_t* ids = d_rowids ? d_rowids : (uint32_t*)((char*)d_ws + stage_off);
   const int64_t cap = d_rowids ? out_cap : (out_cap < n ? out_cap : n);

@@ -324,15 +324,13 @@ int launch_compact(const int32_t* d_key, int64_t n, const SelMasks& mk, const in
     P.eb[j] = j < g.m ? g.elem_bytes[j] : 4;
     P.vec[j] = j < g.m && (((uintptr_t)g.col[j] - (uintptr_t)P.mis * (uintptr_t)g.elem_bytes[j]) & 15u) == 0;
   }
-  static bool attr_set[64] = {};
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 0 && dev < 64 && !attr_set[dev]) {
+  static std::atomic<int> attr_set[64];
+  const int a = device_once(attr_set, current_device(), [] {
     cudaError_t e = cudaFuncSetAttribute(compact_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)sizeof(CtSmem));
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(compact smem)");
-    attr_set[dev] = true;
-  }
+    return e != cudaSuccess ? cuda_fail(e, "cudaFuncSetAttribute(compact smem)") : 1;
+  });
+  if (a < 0) return a;
   const int64_t ntiles = (n + P.mis + SEL_TILE - 1) / SEL_TILE;
   int64_t grid = (int64_t)num_sms() * 2;  // 2 CTAs per SM (launch bounds, ~100 KB of ring each)
   if (grid > ntiles) grid = ntiles;

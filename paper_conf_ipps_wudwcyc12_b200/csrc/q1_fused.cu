@@ -431,8 +431,8 @@ __global__ void __launch_bounds__(Q1T_NT + 32, 1) q1_tma_kernel(const Q1Params P
   reduce_and_fold<Q1T_NW>(A, P, S.s_w, &S.status, &S.last);
 }
 
-int g_q1_occ[64];     // blocks/SM of the grid kernel per device (0 = unknown)
-bool g_q1_attr[64];   // dynamic smem opt-in done for the TMA kernel
+std::atomic<int> g_q1_occ[64];   // blocks/SM of the grid kernel per device (0 = unknown)
+std::atomic<int> g_q1_attr[64];  // 1: dynamic smem opt-in done for the TMA kernel
 
 // First row h < 16 at which every column is 16-B aligned (flags included),
 // or -1.  `flag_align` = required alignment of the flag columns.
@@ -469,9 +469,7 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
   P.accumulate = accumulate;
   P.counter = (uint32_t*)d_ws;
   P.blocks = (Q1Block*)((char*)d_ws + 256);
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev < 0 || dev >= 64) dev = 0;
+  const int dev = current_device();
   // per-thread 64-bit sums stay exact while rows/thread <= 2^17
   const int64_t sms = num_sms();
 
@@ -480,11 +478,11 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
   if (h16 >= 0 && (n - h16) / Q1T_TILE >= 1) {
     P.head = h16;
     P.ngroups = (n - h16) / Q1T_TILE;
-    if (!g_q1_attr[dev]) {
+    const int a = device_once(g_q1_attr, dev, [] {
       cudaError_t e = cudaFuncSetAttribute(q1_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Q1T_SMEM);
-      if (e != cudaSuccess) return cuda_fail(e, "q1_tma_kernel smem attribute");
-      g_q1_attr[dev] = true;
-    }
+      return e != cudaSuccess ? cuda_fail(e, "q1_tma_kernel smem attribute") : 1;
+    });
+    if (a < 0) return a;
     int64_t grid = sms < P.ngroups ? sms : P.ngroups;
     const int64_t min_grid = (n >> 17) / Q1T_NT + 1;
     if (grid < min_grid) grid = min_grid;
@@ -499,13 +497,13 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
   const int64_t h4 = common_head(c, n, 4);
   P.head = h4 >= 0 ? h4 : n;
   P.ngroups = h4 >= 0 ? (n - h4) / 4 : 0;
-  if (g_q1_occ[dev] == 0) {
-    int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, q1_grid_kernel, Q1G_THREADS, 0);
-    if (e != cudaSuccess) return cuda_fail(e, "occupancy query");
-    g_q1_occ[dev] = occ > 0 ? occ : 1;
-  }
-  int64_t grid = sms * g_q1_occ[dev];
+  const int occ = device_once(g_q1_occ, dev, [] {
+    int o = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, q1_grid_kernel, Q1G_THREADS, 0);
+    return e != cudaSuccess ? cuda_fail(e, "occupancy query") : (o > 0 ? o : 1);
+  });
+  if (occ < 0) return occ;
+  int64_t grid = sms * occ;
   if (grid > Q1_MAX_GRID) grid = Q1_MAX_GRID;
   const int64_t work = P.ngroups > 0 ? P.ngroups : n;
   const int64_t need = (work + Q1G_THREADS - 1) / Q1G_THREADS;

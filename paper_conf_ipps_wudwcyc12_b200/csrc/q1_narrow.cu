@@ -416,7 +416,7 @@ __global__ void __launch_bounds__(256) q1_encode_kernel(const EncParams E) {
   if ((threadIdx.x & 31) == 0 && st) atomicOr(E.status, st);
 }
 
-bool g_qn_attr[64];
+std::atomic<int> g_qn_attr[64];  // 1: dynamic smem opt-in done
 
 }  // namespace
 
@@ -436,14 +436,11 @@ int launch_q1_narrow(const ra_lineitem_narrow& c, int64_t n, int32_t cutoff, ra_
   P.accumulate = accumulate;
   P.counter = (uint32_t*)d_ws;
   P.blocks = (Q1Block*)((char*)d_ws + 256);
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev < 0 || dev >= 64) dev = 0;
-  if (!g_qn_attr[dev]) {
+  const int a = device_once(g_qn_attr, current_device(), [] {
     cudaError_t e = cudaFuncSetAttribute(q1n_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)QN_SMEM);
-    if (e != cudaSuccess) return cuda_fail(e, "q1n_kernel smem attribute");
-    g_qn_attr[dev] = true;
-  }
+    return e != cudaSuccess ? cuda_fail(e, "q1n_kernel smem attribute") : 1;
+  });
+  if (a < 0) return a;
   int64_t grid = (int64_t)num_sms() * QN_CTAS_PER_SM;
   const int64_t need = P.ntiles > 0 ? P.ntiles : 1;
   if (grid > need) grid = need;

@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <mutex>
 #include <utility>
 
 #include "ra.h"
@@ -23,6 +24,27 @@ extern std::atomic<uint64_t> g_launches;
 inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
 
 int num_sms();  // of the current device (cached per device)
+
+// The current CUDA device, clamped to the 64 per-device cache slots.
+int current_device();
+
+// Per-device lazy initialisation (kernel attributes, occupancy, SM count):
+// the first caller computes the value under one process-wide mutex, later
+// callers read it lock-free (acquire/release), so concurrent first calls from
+// several host threads are safe (ra.h: calls are reentrant).  `compute`
+// returns a value > 0, or a negative RA_E_* code (not cached).
+std::mutex& init_mutex();
+template <typename F>
+int device_once(std::atomic<int>* slots, int dev, F&& compute) {
+  int v = slots[dev].load(std::memory_order_acquire);
+  if (v > 0) return v;
+  std::lock_guard<std::mutex> g(init_mutex());
+  v = slots[dev].load(std::memory_order_relaxed);
+  if (v > 0) return v;
+  v = compute();
+  if (v > 0) slots[dev].store(v, std::memory_order_release);
+  return v;
+}
 
 // Launch with programmatic stream serialization (see dev::grid_dep_wait).
 template <typename... Params, typename... Args>

@@ -55,8 +55,8 @@
 // Status words carry a 28-bit launch epoch (header word bumped by the last
 // tile), so stale words of earlier launches read as "not ready": no per-call
 // memset and no second kernel.  The ticket counter is reset by the last CTA to
-// finish.  A workspace must be re-zeroed once per 2^28 launches
-// (ra_workspace_init).
+// finish.  The launch before the tag wraps to 0 clears every status word the
+// workspace has held (header high-water mark), so tags never alias.
 
 #include <stdio.h>
 
@@ -85,9 +85,11 @@ constexpr uint64_t FLAG_A = 1ull << 62;  // tile aggregate published
 constexpr int TAG_SHIFT = 34;
 constexpr uint64_t TAG_MASK = (1ull << 28) - 1;
 
-// header: u32 epoch at word 0, u64 ticket counter at byte 8, u32 done counter at byte 16
+// header: u32 epoch at word 0, u64 ticket counter at byte 8, u32 done counter at
+// byte 16, u64 status-word high-water mark at byte 24
 constexpr int H_EPOCH = 0;
 constexpr int H_DONE = 4;
+constexpr int H_HWM = 6;
 
 constexpr int NW = SEL_THREADS / 32;     // compute warps
 constexpr int WROWS = SEL_TILE / NW;     // contiguous rows owned by a compute warp (1024)
@@ -233,7 +235,7 @@ __device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
 
 template <bool HAS_NE>
 __device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
-  bool k = (uint32_t)(x - P.lo) <= P.span;  // lo <= x <= hi
+  bool k = (uint32_t)x - (uint32_t)P.lo <= P.span;  // lo <= x <= hi (mod-2^32 difference)
   if (HAS_NE) {
 #pragma unroll
     for (int j = 0; j < RA_MAX_PREDS; ++j)
@@ -244,7 +246,7 @@ __device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
 
 template <bool HAS_NE>
 __device__ __forceinline__ bool keep2(int32_t x, const SelParams& P) {
-  bool k = (uint32_t)(x - P.lo2) <= P.span2;
+  bool k = (uint32_t)x - (uint32_t)P.lo2 <= P.span2;
   if (HAS_NE) {
 #pragma unroll
     for (int j = 0; j < RA_MAX_PREDS; ++j)
@@ -596,6 +598,16 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
           *P.d_count = 0;
           if (M == 2) *P.d_count2 = 0;
         }
+        // High-water mark of status words this workspace has carried.  When the
+        // next launch's 28-bit tag wraps to 0, clear all of them: a word left by
+        // a launch exactly 2^28 launches earlier could otherwise read as ready.
+        // (Every CTA of this launch is done with the status words; the next
+        // launch reads them only after this grid completes.)
+        uint64_t* hwm = reinterpret_cast<uint64_t*>(P.hdr + H_HWM);
+        uint64_t h = *hwm;
+        if ((uint64_t)ntiles > h) *hwm = h = (uint64_t)ntiles;
+        if (ntiles > 0 && ((S.epoch + 1) & TAG_MASK) == 0)
+          for (uint64_t w = 0; w < h; ++w) P.status[w] = 0ull;
       }
     }
     return;
@@ -812,15 +824,11 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
   for (; head < i; ++head) write_tile<ROWS, M, SM>(S, P, head, tid);
 }
 
-struct KernelCfg {
-  int grid_per_sm[64][8];
-};
-KernelCfg g_cfg;
-
+// smem opt-in + occupancy of each instantiation, once per device
 template <bool HAS_NE, bool ROWS, int M>
 int ensure_config(int dev, int& per_sm) {
-  int& c = g_cfg.grid_per_sm[dev][(HAS_NE ? 1 : 0) + (ROWS ? 2 : 0) + (M == 2 ? 4 : 0)];
-  if (!c) {
+  static std::atomic<int> cfg[64];
+  const int v = device_once(cfg, dev, [] {
     const int smem = (int)sizeof(SmemFor<M>);
     cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE, ROWS, M>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -829,9 +837,10 @@ int ensure_config(int dev, int& per_sm) {
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE, ROWS, M>, BLOCK, smem);
     if (e != cudaSuccess) return cuda_fail(e, "occupancy(select)");
     if (occ < 1) return fail(RA_E_CUDA, "select kernel does not fit on an SM");
-    c = occ;
-  }
-  per_sm = c;
+    return occ;
+  });
+  if (v < 0) return v;
+  per_sm = v;
   return RA_OK;
 }
 
@@ -854,9 +863,7 @@ size_t sel_inter_bytes(int64_t n) {
 }
 
 int sel_ctas_per_sm() {
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev < 0 || dev >= 64) dev = 0;
+  const int dev = current_device();
   int per_sm = 0;
   if (ensure_config<false, false, 1>(dev, per_sm)) return -1;
   return per_sm;
@@ -916,9 +923,7 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
     P.ne[0] = 0;
   }
   if (n_max >= ((int64_t)1 << 34)) return fail(RA_E_INVAL, "n=%lld >= 2^34", (long long)n_max);
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev < 0 || dev >= 64) dev = 0;
+  const int dev = current_device();
   const bool ne = P.n_ne > 0 || P.n_ne2 > 0;
   const bool rw = rows != nullptr || masks != nullptr;
   const bool two = second != nullptr;
@@ -975,8 +980,9 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
   }
   // Unfused composition: one pass per predicate, intermediates at the end of
   // the workspace (disjoint from any status words this workspace can hold).
+  // (from the 256-B aligned end: a caller may pass any ws_bytes >= the required size)
   const size_t rel = (((size_t)(n > 0 ? n : 1) * 4 + 255) / 256) * 256;
-  char* inter = (char*)d_ws + ws_bytes - sel_inter_bytes(n);
+  char* inter = (char*)d_ws + (ws_bytes & ~(size_t)255) - sel_inter_bytes(n);
   int32_t* buf[2] = {(int32_t*)inter, (int32_t*)(inter + rel)};
   int64_t* cnt = (int64_t*)(inter + 2 * rel);
   const int32_t* src = d_in;

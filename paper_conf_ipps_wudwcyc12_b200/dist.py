@@ -4,11 +4,14 @@ The paper runs on one GPU (Table II); sharding is this build's
 extension.  Each rank owns a contiguous row range; the only collectives are
 
 * SELECT: all_gather of one int64 count per rank -> exclusive scan -> the
-  rank's global output offset (outputs stay sharded at known positions);
+  rank's global output offset (outputs stay sharded at known positions).  For
+  device tensors the scan is libra.so's ``ra_select_offsets`` kernel (stream
+  ordered, no host round trip); for host tensors it is plain integer code;
 * Q1: all_gather of the 400-byte ``ra_q1_partial`` of each rank (NCCL has no
   128-bit sum), merged exactly by ``ra_q1_finalize``.
 
-torch.distributed is plumbing only (NCCL on the GPU box, gloo in CPU tests).
+torch.distributed is plumbing only (NCCL on the GPU box, gloo in CPU tests and
+in the 2-rank tests that share one GPU).
 """
 from __future__ import annotations
 
@@ -36,19 +39,46 @@ def exclusive_offsets(counts) -> list[int]:
     return out
 
 
-def exchange_counts(count, group=None, counts=None):
-    """all_gather one int64 count per rank; returns (counts tensor, this rank's
-    global offset, total) — the SELECT exchange (a9).  ``counts`` (int64[world],
-    optional) receives the gathered counts."""
+def _all_gather(out, inp, group=None):
+    """all_gather_into_tensor; gloo with device tensors is staged through host
+    memory (gloo is the CPU-test / shared-GPU functional backend only)."""
+    import torch.distributed as dist
+    if inp.is_cuda and dist.get_backend(group) == "gloo":
+        tmp = out.cpu()
+        dist.all_gather_into_tensor(tmp, inp.cpu(), group=group)
+        out.copy_(tmp)
+    else:
+        dist.all_gather_into_tensor(out, inp, group=group)
+    return out
+
+
+def exchange_counts(count, group=None, counts=None, offsets=None, total=None):
+    """all_gather one int64 count per rank, then the exclusive scan.
+
+    Returns ``(counts, offset, total)``: the gathered counts (int64[world]),
+    this rank's global output offset and the global count.  Device tensors
+    stay on the device (0-dim views, not synchronised); ``counts``,
+    ``offsets`` (int64[world]) and ``total`` (int64[1]) may be preallocated."""
     import torch
     import torch.distributed as dist
     world = dist.get_world_size(group)
-    if counts is None:
-        counts = torch.empty(world, dtype=torch.int64, device=count.device)
-    dist.all_gather_into_tensor(counts, count.reshape(1).to(torch.int64), group=group)
-    offs = torch.cumsum(counts, 0) - counts
     rank = dist.get_rank(group)
-    return counts, offs[rank], counts.sum()
+    dev = count.device
+    if counts is None:
+        counts = torch.empty(world, dtype=torch.int64, device=dev)
+    _all_gather(counts, count.reshape(1).to(torch.int64), group)
+    if counts.is_cuda:
+        from . import _ra
+        if offsets is None:
+            offsets = torch.empty(world, dtype=torch.int64, device=dev)
+        if total is None:
+            total = torch.empty(1, dtype=torch.int64, device=dev)
+        _ra.ra_select_offsets(counts.data_ptr(), world, offsets.data_ptr(), total.data_ptr(),
+                              int(torch.cuda.current_stream(dev).cuda_stream))
+        return counts, offsets[rank], total[0]
+    host = [int(c) for c in counts.tolist()]
+    offs = exclusive_offsets(host)
+    return counts, torch.tensor(offs[rank], dtype=torch.int64), torch.tensor(sum(host), dtype=torch.int64)
 
 
 def gather_partials(partial, group=None):
@@ -57,5 +87,4 @@ def gather_partials(partial, group=None):
     import torch.distributed as dist
     world = dist.get_world_size(group)
     out = torch.empty(world * partial.numel(), dtype=torch.uint8, device=partial.device)
-    dist.all_gather_into_tensor(out, partial, group=group)
-    return out
+    return _all_gather(out, partial, group)

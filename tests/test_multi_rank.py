@@ -103,3 +103,21 @@ def test_two_rank_exchange_and_merge():
     assert all(r[2] for r in res), res
     counts = res[0][4]
     assert [r[3] for r in res] == [0, counts[0]]
+
+
+def test_bench_refuses_world_size_mismatch():
+    """Under torchrun the world size must equal --gpus (else bench.py would time
+    a different number of GPUs than its line claims)."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "1"], capture_output=True,
+                       text=True, timeout=120, env=env)
+    assert r.returncode != 0 and "WORLD_SIZE=2 but --gpus 1" in r.stderr
+
+
+def test_exchange_counts_host_scan():
+    """exchange_counts on host tensors uses plain integer code for the scan."""
+    assert rdist.exclusive_offsets([]) == []
+    assert rdist.exclusive_offsets([2**40, 1, 0]) == [0, 2**40, 2**40 + 1]

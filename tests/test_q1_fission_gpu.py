@@ -107,3 +107,35 @@ def test_first_call_on_a_fresh_workspace(R):
         assert rc == R.RA_OK
         assert [(r["returnflag"], r["linestatus"], r["count_order"], r["sum_charge"]) for r in rows] == \
                [(e["returnflag"], e["linestatus"], e["count_order"], e["sum_charge"]) for e in exp]
+
+
+def test_bench_configuration_fresh_workspaces(R):
+    """Round 1 saw one bench run whose wide and narrow Q1-fission results
+    disagreed on first calls on fresh workspaces.  Root cause: the workspace's
+    zero fill ran on the current stream while the fission streams (not ordered
+    after it) had already accumulated chunk partials into the same bytes.
+    bench.py's exact configuration (SF10, wide chunk 2^22 / narrow chunk 2^23,
+    3 streams), a fresh workspace before each of 20 iterations and no host
+    synchronisation in between: every result equals the oracle."""
+    sf = 10
+    n = ragen.rows_for_sf(sf)
+    cols = ragen.lineitem(5, n, ragen.parts_for_sf(sf))
+    exp, st = oracle.q1(cols, CUTOFF)
+    assert st == 0
+    h = pinned(cols)
+    dcols = {k: v.cuda() for k, v in h.items()}
+    enc, est = R.q1_encode(dcols)
+    assert int(est.item()) == 0
+    del dcols
+    hn = {k: v.cpu().pin_memory() for k, v in enc.items()}
+    del enc
+    ss = streams(3)
+    for it in range(20):
+        R._WS.clear()
+        rows, rc = R.q1_finalize(bytes(R.q1_fission_run(h, 1 << 22, ss)))
+        assert rc == R.RA_OK
+        assert_same(rows, exp)
+        R._WS.clear()
+        nrows, nrc = R.q1_finalize(bytes(R.q1_narrow_fission_run(hn, 1 << 23, ss)))
+        assert nrc == R.RA_OK
+        assert_same(nrows, exp)

@@ -197,3 +197,73 @@ def test_more_than_2_pow_31_rows(R):
     rng = np.random.default_rng(0)
     pos = np.concatenate([np.arange(64), rng.integers(0, c, 1 << 16), np.arange(c - 64, c)])
     np.testing.assert_array_equal(out[torch.from_numpy(pos).cuda()].cpu().numpy(), xh[idx[pos]])
+
+
+@pytest.mark.parametrize("extra", [1, 4, 8, 255, 4096 + 3])
+def test_unfused_workspace_larger_than_required(R, extra):
+    """ws_bytes may exceed the required size by any amount (ra.h): the unfused
+    intermediates are placed from the 256-B aligned end, so an odd or
+    non-multiple-of-8 ws_bytes cannot misalign them."""
+    n = 100_003
+    x = torch.from_numpy(ragen.int32_column(55, n)).cuda()
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 3)]
+    exp = oracle.select(x.cpu().numpy(), preds)
+    need = R.ra_select_workspace_bytes(n, 3, 0)
+    ws = torch.zeros(need + extra + 256, dtype=torch.uint8, device="cuda")
+    out = torch.empty(n, dtype=torch.int32, device="cuda")
+    cnt = torch.empty(1, dtype=torch.int64, device="cuda")
+    P = R.make_preds(preds)
+    R.ra_select_chain(x.data_ptr(), n, P, 3, 0, out.data_ptr(), n, cnt.data_ptr(), ws.data_ptr(), need + extra,
+                      int(torch.cuda.current_stream().cuda_stream))
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == exp.size
+    np.testing.assert_array_equal(out[:exp.size].cpu().numpy(), exp)
+
+
+def test_epoch_tag_wrap_clears_stale_status_words(R):
+    """Status words carry a 28-bit launch tag.  A word left by a launch exactly
+    2^28 launches earlier carries the tag the wrapped epoch will use again: the
+    launch before the wrap must clear every word the workspace has held (header
+    high-water mark), so a later, larger launch never reads such a word as a
+    published aggregate.  Simulated by planting the header and stale words."""
+    n_small, n_big = 5 * 8192 + 11, 40 * 8192 + 5
+    ws = torch.zeros(R.ra_select_workspace_bytes(n_big, 1, 1), dtype=torch.uint8, device="cuda")
+    words = ws[256:].view(torch.int64)
+    hdr32, hdr64 = ws[:256].view(torch.int32), ws[:256].view(torch.int64)
+    flag_a, tag_shift = 1 << 62, 34
+    # stale words of "tag 0" (a launch 2^28 launches ago) with bogus aggregates
+    words[:48] = flag_a | (0 << tag_shift) | 1000
+    hdr32[0] = (1 << 28) - 1      # this launch uses the last tag before the wrap
+    hdr64[3] = 48                 # high-water mark: 48 words carried so far
+    preds = [("lt", 0)]
+    sh = int(torch.cuda.current_stream().cuda_stream)
+    P = R.make_preds(preds)
+    for n in (n_small, n_big, n_big):  # tags 2^28-1, then 0 (the wrap), then 1
+        x = torch.from_numpy(ragen.int32_column(n, n)).cuda()
+        out = torch.empty(n, dtype=torch.int32, device="cuda")
+        cnt = torch.empty(1, dtype=torch.int64, device="cuda")
+        R.ra_select_chain(x.data_ptr(), n, P, 1, 1, out.data_ptr(), n, cnt.data_ptr(), ws.data_ptr(), ws.numel(), sh)
+        torch.cuda.synchronize()
+        exp = oracle.select(x.cpu().numpy(), preds)
+        assert int(cnt.item()) == exp.size, n
+        np.testing.assert_array_equal(out[:exp.size].cpu().numpy(), exp)
+    assert int(hdr32[0].item()) == (1 << 28) + 2 and int(hdr64[3].item()) == 48
+
+
+def test_select_rows_workspace_reuse_across_sizes(R):
+    """Tuple SELECT keeps its order masks and staged ids at the END of the
+    workspace: a later call with larger n on the same (bigger) workspace never
+    reads an earlier call's masks as tile status words."""
+    big = 3 << 20
+    R.select_rows(torch.zeros(big, dtype=torch.int32, device="cuda"), [("lt", 0)])
+    for i, n in enumerate([1 << 16, (1 << 20) + 3, 5000, 1 << 21]):
+        key = ragen.int32_column(300 + i, n)
+        pay = ragen.int32_column(400 + i, n)
+        preds = [("lt", -(2**31) + 2**26)]  # ~1.6%: sparse masks (isolated bits)
+        exp_ids = np.flatnonzero(key < -(2**31) + 2**26)
+        ids, outs, cnt = R.select_rows(torch.from_numpy(key).cuda(), preds, [torch.from_numpy(pay).cuda()])
+        torch.cuda.synchronize()
+        c = int(cnt.item())
+        assert c == exp_ids.size
+        np.testing.assert_array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
+        np.testing.assert_array_equal(outs[0][:c].cpu().numpy(), pay[exp_ids])

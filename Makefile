@@ -25,7 +25,13 @@ $(PKG)/libra.so: $(RA_SRCS) $(RA_HDRS)
 	$(NVCC) $(NVFLAGS) -Iinclude -o $@ $(RA_SRCS) -lpthread 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
 	@grep -E "registers|spill" $(PKG)/ptxas.log | sed 's/^ptxas info    ://' | head -40
 
+# diagnostics builds of the product library with extra compile-time flags:
+#   make variant NAME=wd FLAGS=-DRA_MO_WATCHDOG   ->  build/libra_wd.so  (RA_LIB_PATH=...)
+variant: $(RA_SRCS) $(RA_HDRS)
+	mkdir -p build
+	$(NVCC) $(NVFLAGS) $(FLAGS) -Iinclude -o build/libra_$(NAME).so $(RA_SRCS) -lpthread 2> build/ptxas_$(NAME).log || (cat build/ptxas_$(NAME).log; exit 1)
+
 clean:
 	rm -f ragen/libragen.so oracle/liboracle.so $(PKG)/libra.so $(PKG)/ptxas.log
 
-.PHONY: all clean
+.PHONY: all clean variant

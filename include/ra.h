@@ -226,21 +226,20 @@ int ra_q1_finalize(const ra_q1_partial* h_partials, int n_partials, ra_q1_row* h
  * L286-288, "different SELECT operators need to filter the same input data").
  * One fused pass reads the input once, evaluates every output's predicate
  * chain in registers and compacts each output separately (order-preserving;
- * both tile aggregates travel in one look-back status word).  Output o equals
- * ra_select_chain(d_in, chains[o]).  Stream-ordered.
+ * the M tile aggregates travel in ceil(M/2) look-back status words).  Output
+ * o equals ra_select_chain(d_in, chains[o]).  Stream-ordered.
  *
- *  d_in          device int32[n] (4-B aligned)
+ *  d_in          device int32[n] (4-B aligned), n < 2^34
  *  h_chains[o]   host array of ks[o] predicates (0 <= ks[o] <= RA_MAX_PREDS)
  *  M             number of outputs, 1 <= M <= RA_MAX_OUTPUTS
- *  d_outs[o]     device int32[out_caps[o]]
- *  d_counts[o]   device int64: output o's size (the required size)
- *  d_ws          ra_select_multi_workspace_bytes(n) bytes (for M = 1:
- *                ra_select_workspace_bytes(n, RA_MAX_PREDS, 1)), zeroed once;
- *                beyond the select status words it holds per-CTA spill slots
- *                for tiles whose two runs exceed the shared-memory ring
+ *  d_outs[o]     device int32[out_caps[o]] (4-B aligned; may be NULL if
+ *                out_caps[o] == 0)
+ *  d_counts[o]   device int64 (8-B aligned): output o's size (the required size)
+ *  d_ws          ra_select_multi_workspace_bytes(n) bytes, 256-B aligned,
+ *                zeroed once (tile status words only)
  * Rows beyond out_caps[o] are not written (the count is still exact).
- * RA_E_WORKSPACE if ws_bytes is too small. */
-#define RA_MAX_OUTPUTS 2
+ * RA_E_INVAL on a bad argument, RA_E_WORKSPACE if ws_bytes is too small. */
+#define RA_MAX_OUTPUTS 4
 
 size_t ra_select_multi_workspace_bytes(int64_t n);
 

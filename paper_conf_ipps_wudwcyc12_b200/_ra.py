@@ -13,7 +13,9 @@ import os
 import re
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libra.so")
+# RA_LIB_PATH: load a diagnostics build of libra.so (scripts/; e.g. compile-time
+# variants or the watchdog build).  Tests, smoke() and bench.py never set it.
+LIB_PATH = os.environ.get("RA_LIB_PATH") or os.path.join(_HERE, "libra.so")
 HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "ra.h")
 
 if not os.path.exists(LIB_PATH):
@@ -31,7 +33,7 @@ RA_E_CUDA = -5
 RA_E_WORKSPACE = -6
 RA_MAX_PREDS = 8
 RA_MAX_PAYLOAD = 4
-RA_MAX_OUTPUTS = 2
+RA_MAX_OUTPUTS = 4
 RA_MAX_RANKS = 65536
 RA_Q1_GROUPS = 6
 RA_LT, RA_LE, RA_GT, RA_GE, RA_EQ, RA_NE = range(6)

@@ -189,7 +189,7 @@ RA_API int ra_select_chain(const int32_t* d_in, int64_t n, const ra_pred* h_pred
 
 RA_API size_t ra_select_multi_workspace_bytes(int64_t n) {
   if (n < 0) n = 0;
-  return ((ra_select_workspace_bytes(n, RA_MAX_PREDS, 1) + 255) / 256) * 256 + ra::sel_spill_bytes(n);
+  return ra::mo_workspace_bytes(n);
 }
 
 RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const* h_chains, const int* ks, int M,
@@ -197,33 +197,29 @@ RA_API int ra_select_multi(const int32_t* d_in, int64_t n, const ra_pred* const*
                            size_t ws_bytes, ra_stream_t stream) {
   clear_error();
   if (M < 1 || M > RA_MAX_OUTPUTS) return fail(RA_E_INVAL, "M=%d outside [1, %d]", M, RA_MAX_OUTPUTS);
-  if (!h_chains || !ks || !d_outs || !out_caps || !d_counts) return fail(RA_E_INVAL, "null argument");
+  if (!h_chains || !ks || !d_outs || !out_caps || !d_counts || !d_ws) return fail(RA_E_INVAL, "null argument");
+  if (n < 0) return fail(RA_E_INVAL, "negative n");
+  if (n > 0 && !d_in) return fail(RA_E_INVAL, "null d_in with n > 0");
+  if ((uintptr_t)d_in & 3u) return fail(RA_E_INVAL, "d_in must be 4-byte aligned");
+  if ((uintptr_t)d_ws & 255u) return fail(RA_E_INVAL, "workspace must be 256-byte aligned");
+  const size_t need = ra_select_multi_workspace_bytes(n);
+  if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
   CanonPred cp[RA_MAX_OUTPUTS];
   for (int o = 0; o < M; ++o) {
-    int rc = check_select_args(d_in, n, ks[o], d_outs[o], out_caps[o], d_counts[o], d_ws, ws_bytes, 1);
-    if (rc) return rc;
+    if (out_caps[o] < 0) return fail(RA_E_INVAL, "output %d: negative out_cap", o);
+    if (out_caps[o] > 0 && !d_outs[o]) return fail(RA_E_INVAL, "output %d: null d_out with out_cap > 0", o);
+    if (!d_counts[o]) return fail(RA_E_INVAL, "output %d: null d_count", o);
+    if (((uintptr_t)d_outs[o] & 3u) || ((uintptr_t)d_counts[o] & 7u))
+      return fail(RA_E_INVAL, "output %d: misaligned d_out or d_count", o);
+    if (ks[o] < 0 || ks[o] > RA_MAX_PREDS) return fail(RA_E_INVAL, "output %d: k=%d outside [0, %d]", o, ks[o], RA_MAX_PREDS);
     if (ks[o] > 0 && !h_chains[o]) return fail(RA_E_INVAL, "null chain %d with k > 0", o);
     for (int j = 0; j < ks[o]; ++j)
       if (h_chains[o][j].op < RA_LT || h_chains[o][j].op > RA_NE)
         return fail(RA_E_INVAL, "output %d predicate %d: unknown op %d", o, j, (int)h_chains[o][j].op);
-    rc = canonicalize(h_chains[o], ks[o], &cp[o]);
+    int rc = canonicalize(h_chains[o], ks[o], &cp[o]);
     if (rc) return rc;
   }
-  if (M == 1)
-    return launch_select_pass(d_in, n, nullptr, cp[0], d_outs[0], out_caps[0], d_counts[0], d_ws,
-                              (cudaStream_t)stream);
-  SelSecond second;
-  second.cp = cp[1];
-  second.out = d_outs[1];
-  second.out_cap = out_caps[1];
-  second.d_count = d_counts[1];
-  const size_t need = ra_select_multi_workspace_bytes(n);
-  if (ws_bytes < need) return fail(RA_E_WORKSPACE, "workspace %zu < required %zu", ws_bytes, need);
-  // spill slots at the (256-B aligned) END of the workspace: the status words
-  // of a later call on the same workspace with any n never reach them
-  second.spill = (int32_t*)((char*)d_ws + (ws_bytes & ~(size_t)255) - ra::sel_spill_bytes(n));
-  return launch_select_pass(d_in, n, nullptr, cp[0], d_outs[0], out_caps[0], d_counts[0], d_ws, (cudaStream_t)stream,
-                            nullptr, &second);
+  return ra::launch_select_multi(d_in, n, cp, M, d_outs, out_caps, d_counts, d_ws, (cudaStream_t)stream);
 }
 
 RA_API size_t ra_select_rows_workspace_bytes(int64_t n, int k) {

@@ -129,6 +129,12 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
                        cudaStream_t s, uint32_t* rows = nullptr, const SelSecond* second = nullptr,
                        const SelMasks* masks = nullptr);
 
+// Several SELECTs on one input in one pass (select_multi.cu), 1 <= M <= 4:
+// cp[o] = output o's folded chain; validated arguments.
+int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int M, int32_t* const* d_outs,
+                        const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s);
+size_t mo_workspace_bytes(int64_t n);
+
 // Payload fields of a tuple SELECT.  The selectivity decides, on the device,
 // which of the two kernels launched back to back places them: the id gather
 // when count * sparse_den <= n (few rows: read only their sectors), else the

@@ -59,6 +59,7 @@
 // workspace has held (header high-water mark), so tags never alias.
 
 #include <stdio.h>
+#include <stdlib.h>
 
 #include <type_traits>
 
@@ -326,13 +327,26 @@ __device__ __forceinline__ int64_t window_sum(const SM& S, const SelParams& P, i
   const int64_t lo = S.wlo[q], hi = S.whi[q];
   const int64_t s0 = lo & ~1ll;
   const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
+  const uint64_t pad = (uint64_t)want << 32;  // a ready word with a zero aggregate
   int64_t total = 0;
+  // lane l takes words base + l + 32c: conflict-free shared loads, and on the
+  // copied path no branches (clamped addresses + selects)
   for (int64_t base = lo; base < hi; base += PASS_WORDS) {
     uint64_t w[LBW];
+    if (copied) {
 #pragma unroll
-    for (int c = 0; c < LBW; ++c) {
-      const int64_t idx = base + LBW * lane + c;  // tile whose aggregate this word is
-      w[c] = idx >= hi ? ((uint64_t)want << 32) : copied ? S.win[q][idx - s0] : dev::ld_relaxed_u64(P.status + idx);
+      for (int c = 0; c < LBW; ++c) {
+        const int64_t idx = base + lane + 32 * c;
+        const bool in = idx < hi;
+        const uint64_t x = S.win[q][(in ? idx : lo) - s0];
+        w[c] = in ? x : pad;
+      }
+    } else {
+#pragma unroll
+      for (int c = 0; c < LBW; ++c) {
+        const int64_t idx = base + lane + 32 * c;
+        w[c] = idx < hi ? dev::ld_relaxed_u64(P.status + idx) : pad;
+      }
     }
     for (int spins = 0;; ++spins) {
       bool missing = false;
@@ -343,7 +357,7 @@ __device__ __forceinline__ int64_t window_sum(const SM& S, const SelParams& P, i
       if (spins > 1) __nanosleep(64);
 #pragma unroll
       for (int c = 0; c < LBW; ++c)
-        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + LBW * lane + c);
+        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + lane + 32 * c);
     }
     uint32_t v = 0;
 #pragma unroll
@@ -361,13 +375,24 @@ __device__ __forceinline__ void window_sum2(const SM& S, const SelParams& P, int
   const int64_t lo = S.wlo[q], hi = S.whi[q];
   const int64_t s0 = lo & ~1ll;
   const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
+  const uint64_t pad = (uint64_t)want << 32;
   t0 = t1 = 0;
   for (int64_t base = lo; base < hi; base += PASS_WORDS) {
     uint64_t w[LBW];
+    if (copied) {
 #pragma unroll
-    for (int c = 0; c < LBW; ++c) {
-      const int64_t idx = base + LBW * lane + c;
-      w[c] = idx >= hi ? ((uint64_t)want << 32) : copied ? S.win[q][idx - s0] : dev::ld_relaxed_u64(P.status + idx);
+      for (int c = 0; c < LBW; ++c) {
+        const int64_t idx = base + lane + 32 * c;
+        const bool in = idx < hi;
+        const uint64_t x = S.win[q][(in ? idx : lo) - s0];
+        w[c] = in ? x : pad;
+      }
+    } else {
+#pragma unroll
+      for (int c = 0; c < LBW; ++c) {
+        const int64_t idx = base + lane + 32 * c;
+        w[c] = idx < hi ? dev::ld_relaxed_u64(P.status + idx) : pad;
+      }
     }
     for (int spins = 0;; ++spins) {
       bool missing = false;
@@ -377,7 +402,7 @@ __device__ __forceinline__ void window_sum2(const SM& S, const SelParams& P, int
       if (spins > 1) __nanosleep(64);
 #pragma unroll
       for (int c = 0; c < LBW; ++c)
-        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + LBW * lane + c);
+        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + lane + 32 * c);
     }
     uint32_t v0 = 0, v1 = 0;
 #pragma unroll
@@ -945,6 +970,10 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
   int64_t grid = (int64_t)num_sms() * per_sm;
   if (two && grid > SEL_MULTI_MAX_GRID) grid = SEL_MULTI_MAX_GRID;  // spill slots exist for this many CTAs
+  // RA_SEL_MAX_CTAS (diagnostics only): cap the grid, for the paper's Fig 12
+  // experiment (a SELECT with half the CTAs, two of them on two streams)
+  static const int64_t max_ctas = getenv("RA_SEL_MAX_CTAS") ? atoll(getenv("RA_SEL_MAX_CTAS")) : 0;
+  if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
   if (grid > ntiles_max) grid = ntiles_max;
   if (grid < 1) grid = 1;
   // No co-residency is required (plain launch): a CTA only ever waits on the

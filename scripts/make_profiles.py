@@ -28,6 +28,20 @@ CAPTURES = {  # report -> (summary name, traffic key, command)
     "prof_q1n": ("q1n_sf10", "q1n_sf10", "python scripts/prof_driver.py q1n 5  (SF10 narrow, 60M rows)"),
     "prof_compact": ("compact_k2_s05_n28", "compact_k2_s0.5_n28",
                      "python scripts/prof_driver.py rows 5  (payload compaction of 3 int32 fields, 2^28 rows, k=2, s=0.5/stage)"),
+    "prof_q1_sf100": ("q1_sf100", "q1_sf100", "python scripts/prof_driver.py q1sf100 3  (SF100, 600M rows, one GPU)"),
+    "prof_q1n_sf100": ("q1n_sf100", "q1n_sf100", "python scripts/prof_driver.py q1nsf100 3  (SF100 narrow, 600M rows)"),
+    "prof_multi": ("select_multi_m2_s05_n28", "select_multi_m2_s0.5_n28",
+                   "python scripts/prof_driver.py multi 5 28 2  (2^28 int32, 2 outputs: x<0 | -2^30<x<2^30)"),
+    "prof_multi_dense": ("select_multi_m2_s09_n28", "select_multi_m2_s0.9_n28",
+                         "python scripts/prof_driver.py multi 5 28 2 0.9  (2^28 int32, 2 outputs keeping ~90% each)"),
+    "prof_multi4": ("select_multi_m4_n28", "select_multi_m4_n28",
+                    "python scripts/prof_driver.py multi 5 28 4  (2^28 int32, 4 outputs: .5 .5 .25 .25)"),
+    "prof_sparse_sel": ("sparse_select_k1_s001_n28", "sparse_select_k1_s0.01_n28",
+                        "python scripts/prof_driver.py sparse 5 28 1 0.01  (key pass of the sparse tuple SELECT)"),
+    "prof_sparse_ids": ("sparse_ids_k1_s001_n28", "sparse_ids_k1_s0.01_n28",
+                        "python scripts/prof_driver.py sparse 5 28 1 0.01  (ids_kernel: row ids from the order masks)"),
+    "prof_sparse_gather": ("sparse_gather_k1_s001_n28", "sparse_gather_k1_s0.01_n28",
+                           "python scripts/prof_driver.py sparse 5 28 1 0.01  (gather_kernel: 3 int32 fields at the ids)"),
 }
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
@@ -88,3 +102,30 @@ if os.path.exists(lpath):
         lines.append(f"{len(v):4d}  {sum(v) / len(v):12.0f}  {sum(v) / total * 100:5.1f}%  {k[:110]}")
     open(os.path.join(OUT, f"r{RND}_launches.txt"), "w").write("\n".join(lines) + "\n")
     print("wrote launches")
+
+# PCIe bytes of the fission paths (ncu application-range replay of scripts/pcie_ranges.py)
+ppath = os.path.join(ROOT, "gpurun_out", "pcie.csv")
+if os.path.exists(ppath):
+    rows = [r for r in csv.reader(open(ppath)) if len(r) > 5]
+    h = rows[0]
+    ii, mi, ui, vi = h.index("ID"), h.index("Metric Name"), h.index("Metric Unit"), h.index("Metric Value")
+    names = ["select_fission_n28", "select_fission_n30", "q1_fission_sf10", "q1n_fission_sf10"]
+    per = collections.OrderedDict()
+    for r in rows[1:]:
+        per.setdefault(int(r[ii]), {})[r[mi]] = (r[vi], r[ui])
+    pcie = {}
+    lines = [f"# round {RND}: ncu --replay-mode app-range --profile-from-start off --metrics "
+             "pcie__read_bytes.sum,pcie__write_bytes.sum,gpu__time_duration.sum python scripts/pcie_ranges.py",
+             "# one range = one synchronous fission call (H2D + kernels + D2H); read = host->device over PCIe",
+             "# range                    pcie_read_bytes   pcie_write_bytes   range_ms   read GB/s"]
+    for (rid, m), name in zip(sorted(per.items()), names):
+        rd = to_bytes(*m["pcie__read_bytes.sum"]) if "pcie__read_bytes.sum" in m else float("nan")
+        wr = to_bytes(*m["pcie__write_bytes.sum"]) if "pcie__write_bytes.sum" in m else float("nan")
+        t, tu = m.get("gpu__time_duration.sum", ("nan", "ns"))
+        ns = float(t.replace(",", "")) * {"ns": 1, "us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6,
+                                           "nsecond": 1}.get(tu, 1)
+        pcie[name] = {"pcie_read_bytes": rd, "pcie_write_bytes": wr, "range_ns": ns}
+        lines.append(f"{name:24s} {rd:17.0f} {wr:18.0f} {ns / 1e6:10.3f} {rd / ns if ns else 0:10.1f}")
+    json.dump(pcie, open(os.path.join(OUT, "ncu_pcie.json"), "w"), indent=1, sort_keys=True)
+    open(os.path.join(OUT, f"r{RND}_pcie.txt"), "w").write("\n".join(lines) + "\n")
+    print("wrote pcie")

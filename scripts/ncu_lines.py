@@ -9,7 +9,9 @@ N = int(sys.argv[4]) if len(sys.argv) > 4 else 30
 d = tempfile.mkdtemp()
 subprocess.run(["cuobjdump", "-xelf", "all", os.path.abspath("paper_conf_ipps_wudwcyc12_b200/libra.so")], cwd=d,
                capture_output=True)
-cub = [f for f in os.listdir(d) if os.path.basename(srcfile).split('.')[0] in f and f.endswith(".cubin")][0]
+stem = os.path.basename(srcfile).split('.')[0]
+cands = sorted(f for f in os.listdir(d) if stem in f and f.endswith(".cubin"))
+cub = next((f for f in cands if f == stem + ".sm_100a.cubin"), cands[0])
 sass = subprocess.run(["nvdisasm", "--print-line-info", os.path.join(d, cub)], capture_output=True, text=True).stdout
 blocks = re.split(r"//-+ \.text\.", sass)
 blk = [b for b in blocks if kname in b.split("\n")[0]][0]

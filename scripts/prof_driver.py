@@ -1,6 +1,7 @@
 """Small driver for ncu: runs the hot-path kernels a few times at bench sizes.
 
-usage: python scripts/prof_driver.py {select|unfused|rows|q1|q1n|q1time|select1m} [reps] [log2n] [k] [sel]
+usage: python scripts/prof_driver.py {select|unfused|rows|sparse|multi|q1|q1sf100|q1n|q1nsf100|q1time|select1m}
+       [reps] [log2n] [k] [sel]
 """
 import os
 import sys
@@ -79,13 +80,47 @@ def main():
         enc, _ = R.q1_encode(cols)
         for _ in range(reps):
             R.q1_narrow(enc)
-    elif what == "q1":
-        n = ragen.rows_for_sf(10)
+    elif what in ("q1", "q1sf100", "q1nsf100"):
+        sf = 10 if what == "q1" else 100
+        n = ragen.rows_for_sf(sf)
         cols = {name: torch.empty(n, dtype=getattr(torch, np.dtype(dt).name), device="cuda")
                 for name, dt in ragen.LINEITEM_COLUMNS}
-        ragen.lineitem_dev(5, ragen.parts_for_sf(10), cols)
+        ragen.lineitem_dev(5, ragen.parts_for_sf(sf), cols)
+        if what == "q1nsf100":
+            cols, _ = R.q1_encode(cols)
+            torch.cuda.empty_cache()
         for _ in range(reps):
-            R.q1(cols)
+            (R.q1_narrow if what == "q1nsf100" else R.q1)(cols)
+    elif what == "multi1":  # the multi kernel with one output (M = 1) at selectivity sel
+        n = 1 << log2n
+        x = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(2, x)
+        ch = [[("lt", ragen.nested_thresholds(sel, 1)[0])]]
+        out = torch.empty(n, dtype=torch.int32, device="cuda")
+        for _ in range(reps):
+            R.select_multi(x, ch, outs=[out])
+    elif what == "multi":  # f2: M outputs on one 2^log2n column, the bench's chains (M = k arg)
+        n = 1 << log2n
+        x = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(2, x)
+        chains = [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)], [("ge", 2**30)], [("lt", -(2**30))]][:k]
+        if sel > 0.5:  # dense pair: both outputs keep ~sel
+            t = int(-(2**31) + sel * 2**32)
+            chains = [[("lt", t)], [("gt", -t)]][:k]
+        outs = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in chains]
+        for _ in range(reps):
+            R.select_multi(x, chains, outs=outs)
+    elif what == "sparse":  # f3 sparse path: 3 int32 fields at s=0.01 (ids_kernel + gather_kernel)
+        n = 1 << log2n
+        x = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(2, x)
+        f1 = torch.empty(n, dtype=torch.int32, device="cuda")
+        f2 = torch.empty(n, dtype=torch.int32, device="cuda")
+        ragen.int32_column_dev(102, f1)
+        ragen.int32_column_dev(103, f2)
+        preds = [("lt", t) for t in ragen.nested_thresholds(sel, k)]
+        for _ in range(reps):
+            R.select_rows(x, preds, [x, f1, f2], rowids=False)
     torch.cuda.synchronize()
     print("done", what)
 

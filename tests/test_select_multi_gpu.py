@@ -5,6 +5,7 @@ tiles, every selectivity regime, != predicates, capacity limits, and
 interleaved with single-output calls on the same workspace."""
 import numpy as np
 import pytest
+from hypothesis import given, settings, strategies as st
 
 import oracle
 import ragen
@@ -36,7 +37,7 @@ def check(R, x, chains, offset=0):
 def test_sizes_offsets(R, n, offset):
     x = ragen.int32_column(71 + n, n)
     check(R, x, [[("lt", 0)], [("gt", -(2**29)), ("lt", 2**30)]], offset)
-    check(R, x, [[("gt", -(2**31) + 2**28)], [("ne", 7)]], offset)  # both dense: spilled second runs
+    check(R, x, [[("gt", -(2**31) + 2**28)], [("ne", 7)]], offset)  # both dense
 
 
 @pytest.mark.parametrize("s0,s1", [(0.0, 1.0), (0.01, 0.9), (0.5, 0.5), (0.9, 0.9), (1.0, 1.0), (0.25, 0.75)])
@@ -92,7 +93,7 @@ def test_capacity(R):
 @pytest.mark.parametrize("caps", [(1000, 5), (3 * 8192 + 17, 10**9), (0, 123457)])
 def test_capacity_dense_outputs(R, caps):
     """Both outputs keep ~90% of every tile, more than the selected-row ring
-    holds: those tiles are placed straight from registers; truncation stays exact
+    holds at once: compaction waits for the writers; truncation stays exact
     and nothing is written past either capacity."""
     n = 50 * 8192 + 99
     x = ragen.int32_column(76, n)
@@ -124,8 +125,85 @@ def test_capacity_dense_outputs(R, caps):
 def test_argument_errors(R):
     xd = torch.zeros(16, dtype=torch.int32, device="cuda")
     with pytest.raises(R.RAError) as e:
-        R.select_multi(xd, [[("lt", 0)]] * 3)
+        R.select_multi(xd, [[("lt", 0)]] * (R.RA_MAX_OUTPUTS + 1))
     assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:
+        R.select_multi(xd, [[("lt", 0)], [(7, 0)]])
+    assert e.value.code == R.RA_E_INVAL
+
+
+def _chain(s):
+    if s == 0.0:
+        return [("lt", -(2**31))]
+    if s == 1.0:
+        return [("ge", -(2**31))]
+    return [("lt", ragen.nested_thresholds(s, 1)[0])]
+
+
+@pytest.mark.parametrize("n", [0, 1, 5, 4095, 4096, 4097, 7 * 4096 + 1234, 1_000_003])
+@pytest.mark.parametrize("offset", [0, 3])
+@pytest.mark.parametrize("M", [3, 4])
+def test_three_four_outputs_sizes_offsets(R, n, offset, M):
+    x = ragen.int32_column(171 + n, n)
+    chains = [[("lt", 0)], [("gt", -(2**29)), ("lt", 2**30)], [("ne", int(x[0]) if n else 3)], [("ge", 2**30)]][:M]
+    check(R, x, chains, offset)
+
+
+@pytest.mark.parametrize("sel", [(0.0, 0.0, 0.0, 0.0), (1.0, 1.0, 1.0, 1.0), (0.9, 0.9, 0.9, 0.9),
+                                 (0.01, 0.5, 0.99, 0.25), (0.5, 0.5, 0.5), (1.0, 0.0, 1.0), (0.9, 0.9)])
+def test_many_outputs_selectivities_many_tiles(R, sel):
+    """Up to four outputs, every one dense (a tile's M runs fill most of the
+    ring), empty, or mixed; 2^22+ rows = hundreds of tiles per SM."""
+    n = (1 << 22) + 333
+    x = ragen.int32_column(172, n)
+    check(R, x, [_chain(s) for s in sel])
+
+
+@settings(max_examples=40, deadline=None)
+@given(st.integers(1, 4), st.integers(0, 70000), st.integers(0, 3), st.data())
+def test_random_chains_brute_force(R, M, n, offset, data):
+    """Random predicate chains (all six ops, up to 8 per output) on random
+    data; each output vs the oracle (itself pinned by brute force)."""
+    rng = np.random.default_rng(n * 7 + M)
+    x = rng.integers(-50, 50, n, dtype=np.int32) if n % 2 else rng.integers(-(2**31), 2**31, n, dtype=np.int64).astype(np.int32)
+    ops = ["lt", "le", "gt", "ge", "eq", "ne"]
+    chains = []
+    for _ in range(M):
+        k = data.draw(st.integers(0, 8))
+        chains.append([(data.draw(st.sampled_from(ops)), data.draw(st.integers(-60, 60))) for _ in range(k)])
+    check(R, x, chains, offset)
+
+
+def test_workspace_shared_across_output_counts(R):
+    """One workspace, successive launches with M = 1..4 (tile size 8192 for
+    M <= 2, 4096 for M >= 3: different status-word layouts on the same words)."""
+    n = 3 * (1 << 20) + 11
+    x = ragen.int32_column(174, n)
+    xd = torch.from_numpy(x).cuda()
+    chains = [[("lt", 0)], [("gt", -(2**30))], [("ne", 5), ("lt", 2**30)], [("ge", -(2**29))]]
+    exp = oracle.select_multi(x, chains)
+    for M in (4, 1, 3, 2, 4, 4, 1, 2, 3):
+        outs, cnt = R.select_multi(xd, chains[:M])
+        torch.cuda.synchronize()
+        for o in range(M):
+            c = int(cnt[o].item())
+            assert c == exp[o].size, (M, o)
+            assert np.array_equal(outs[o][:c].cpu().numpy(), exp[o]), (M, o)
+
+
+def test_full_size_four_outputs(R):
+    """2^28 device-generated rows (seed 2), four outputs (.5, .5, .25, .25):
+    the bench's M = 4 shape, full comparison with the oracle."""
+    n = 1 << 28
+    x = torch.empty(n, dtype=torch.int32, device="cuda")
+    ragen.int32_column_dev(2, x)
+    chains = [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)], [("ge", 2**30)], [("lt", -(2**30))]]
+    outs, cnt = R.select_multi(x, chains)
+    torch.cuda.synchronize()
+    exp = oracle.select_multi(x.cpu().numpy(), chains)
+    for o, c, e in zip(outs, cnt.cpu().tolist(), exp):
+        assert int(c) == e.size
+        np.testing.assert_array_equal(o[:int(c)].cpu().numpy(), e)
 
 
 def test_full_size_bench_config(R):
@@ -148,7 +226,7 @@ def test_two_outputs_past_2_pow_31_rows_closed_form(R):
     """n = 2^31 + 2^28 rows with key[i] = int32(i) (wrapping): output 0 keeps
     key >= 0 (rows 0 .. 2^31-1: 2^31 outputs, the last at position 2^31 - 1),
     output 1 keeps key < 2^30 (rows 0 .. 2^30-1, then the wrapped rows 2^31 ..
-    n-1); while both keep whole tiles the second run spills.  Counts exact,
+    n-1); both outputs keep whole tiles for 2^30 rows.  Counts exact,
     sampled outputs against the closed form."""
     n = (1 << 31) + (1 << 28)
     x = torch.empty(n, dtype=torch.int32, device="cuda")

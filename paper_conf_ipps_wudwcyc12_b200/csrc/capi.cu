@@ -144,7 +144,10 @@ RA_API int ra_workspace_init(void* d_ws, size_t ws_bytes, ra_stream_t stream) {
 
 RA_API size_t ra_select_workspace_bytes(int64_t n, int k, int fused) {
   if (n < 0) n = 0;
+  // status words of either pass kind (the fused chain runs the multi-output
+  // pass, the unfused composition's passes the single-output kernel)
   size_t b = (sel_status_bytes(n) + 255) / 256 * 256;
+  if (ra::mo_workspace_bytes(n) > b) b = ra::mo_workspace_bytes(n);
   if (!fused && k > 1) b += sel_inter_bytes(n);
   return b;
 }

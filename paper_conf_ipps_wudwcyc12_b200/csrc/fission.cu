@@ -108,7 +108,8 @@ RA_API int ra_fission_run(const int32_t* h_in, int64_t n, const ra_pred* h_preds
   // workspace can never read as tile status.
   for (int s = 0; s < S; ++s) {
     char* base = (char*)d_ws + (size_t)s * per;
-    cudaError_t e = cudaMemsetAsync(base + 2 * io, 0, sel_status_bytes(chunk_rows), (cudaStream_t)streams[s]);
+    cudaError_t e = cudaMemsetAsync(base + 2 * io, 0, ra_select_workspace_bytes(chunk_rows, 1, 1),
+                                    (cudaStream_t)streams[s]);
     if (e != cudaSuccess) {
       for (int j = 0; j < S; ++j) cudaEventDestroy(ev[j]);
       return cuda_fail(e, "cudaMemsetAsync(fission control words)");

@@ -1002,10 +1002,12 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
                       int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
                       size_t ws_bytes, cudaStream_t s) {
   if (fused || k <= 1) {
+    // the fused chain is one output of the warp-specialised multi-output pass
+    // (select_multi.cu): one kernel, writer warps, cooperative look-back
     CanonPred cp;
     int rc = canonicalize(h_preds, k, &cp);
     if (rc) return rc;
-    return launch_select_pass(d_in, n, nullptr, cp, d_out, out_cap, d_count, d_ws, s, nullptr);
+    return launch_select_multi(d_in, n, &cp, 1, &d_out, &out_cap, &d_count, d_ws, s);
   }
   // Unfused composition: one pass per predicate, intermediates at the end of
   // the workspace (disjoint from any status words this workspace can hold).

@@ -33,6 +33,8 @@
 // its high half carries this launch's tag, so no per-call memset (select_fused
 // uses the same scheme; see there for the look-back's lag and windows).
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <stdio.h>
 #include <string.h>
 
@@ -52,32 +54,48 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 #define RA_MO_NG 2  // compute groups per CTA
 #endif
 #ifndef RA_MO_NWR
-#define RA_MO_NWR 2  // writer warps per CTA
+#define RA_MO_NWR 4  // writer warps per CTA (aux warps fill whole warpgroups)
+#endif
+#ifndef RA_MO_REGS
+// setmaxnreg: the compute warpgroups run with RA_MO_REGS registers, the aux
+// warpgroups (look-back, producer, writers) with RA_MO_AUXREGS; an increase is
+// served only from what this CTA's decreases released (0: no rebalancing)
+#define RA_MO_REGS 88
+#define RA_MO_AUXREGS 56
+#endif
+#ifndef RA_MO_TMA
+#define RA_MO_TMA 0  // writer: TMA bulk tensor stores instead of warp stores
+#endif
+#ifndef RA_MO_WU
+#define RA_MO_WU 8  // writer: ring loads in flight per lane
 #endif
 #ifndef RA_MO_D1
-#define RA_MO_D1 1  // window of tile k copied once tile k+D1 is counted (or on demand)
+// window of tile k copied once tile k+D1 is counted (or on demand); measured
+// best: 2 for one output (the words before a tile are older), 1 for several
+// (dense runs wait for the ring sooner)
+#define RA_MO_D1 0
 #endif
 #ifndef RA_MO_IN_KB
 #define RA_MO_IN_KB 96  // input ring per CTA
 #endif
 constexpr int NG = RA_MO_NG;
 constexpr int NWR = RA_MO_NWR;
-constexpr int D1 = RA_MO_D1;
 constexpr int GW = 8;                         // warps per compute group
 constexpr int GT = 32 * GW;                   // threads per compute group
 constexpr int NCW = NG * GW;                  // compute warps
-constexpr int LBWARP = NCW, PRWARP = NCW + 1, WR0 = NCW + 2;
-constexpr int BLOCK = 32 * (NCW + 2 + NWR);
+#ifndef RA_MO_NLB
+#define RA_MO_NLB 3  // look-back warps
+#endif
+constexpr int NLB = RA_MO_NLB;
+constexpr int LBWARP = NCW, PRWARP = NCW + NLB, WR0 = NCW + NLB + 1;
+constexpr int BLOCK = 32 * (NCW + NLB + 1 + NWR);
 #ifndef RA_MO_K
 #define RA_MO_K 8
 #endif
 constexpr int K = RA_MO_K;                    // metadata slots: tiles counted but not yet written
 constexpr int LBW = 10;                       // status words per look-back lane per pass
 constexpr int PASS_WORDS = 32 * LBW;
-#ifndef RA_MO_Q
-#define RA_MO_Q 4  // look-back windows in flight
-#endif
-constexpr int Q = RA_MO_Q;
+constexpr int Q = NLB;                        // window slots: one per look-back warp
 constexpr int WIN_WORDS = 512;                // window slot (status words)
 constexpr int SMEM_BUDGET = 232448;           // max dynamic shared memory per CTA on sm_100
 
@@ -90,11 +108,18 @@ struct Cfg {
   static constexpr int NPK = VEC / 4;                // packed 8-bit count words per lane per output
   static constexpr int W = (M + 1) / 2;              // status words per tile
   static constexpr int INSLOTS = RA_MO_IN_KB * 1024 / (TILE * 4);
+  static constexpr int D1 = RA_MO_D1 > 0 ? RA_MO_D1 : (M == 1 ? 2 : 1);
 };
 __host__ __device__ constexpr int q_of(int npk, int j) { return npk == 2 ? (j & 1) : 0; }
 __host__ __device__ constexpr int b_of(int npk, int j) { return npk == 2 ? (j >> 1) : ((j >> 1) | ((j & 1) << 1)); }
 
 struct MoParams {
+  // per output: 1-D TMA maps of the output (int32, element coordinates from
+  // its 16-B aligned base, bounded by out_cap: the copy engine clips rows past
+  // the capacity) with boxes of 256 and 32 rows; tma[o] = 0: plain stores
+  CUtensorMap tmap[RA_MAX_OUTPUTS][2];
+  int32_t tma[RA_MAX_OUTPUTS];
+  int32_t omis[RA_MAX_OUTPUTS];  // rows of out[o]'s 16-B chunk before out[o]
   const int32_t* abase;  // 16-B aligned base, = d_in - mis
   int64_t n;
   uint32_t* hdr;
@@ -127,6 +152,10 @@ struct MoFixed {  // everything but the ring
   int32_t cnt[K][M];
   int32_t start[K];  // ring position of the tile's first run (runs back to back, output order)
   uint32_t wtot[2 * NG][M][GW];
+  int64_t pfx[M];     // look-back chain: inclusive prefixes after tile chain_done - 1
+  int32_t chain_done; // tiles placed
+  int32_t end_tile;   // the CTA's end-marker tile index (INT32_MAX until known)
+  int32_t lb_done;    // look-back warps finished
   int64_t n;
   uint32_t epoch;
   int32_t demand;
@@ -141,7 +170,7 @@ constexpr int ring_ints() {
 template <int M>
 struct __align__(128) MoSmem : MoFixed<M> {
   static constexpr int RING = ring_ints<M>();
-  int32_t ring[RING];
+  alignas(128) int32_t ring[RING];  // runs start at multiples of 32 rows (128 B): TMA store sources
 };
 static_assert(MoSmem<1>::RING >= 8192 && MoSmem<2>::RING >= 2 * 8192 && MoSmem<3>::RING >= 3 * 4096 &&
                   MoSmem<4>::RING >= 4 * 4096,
@@ -212,6 +241,22 @@ __device__ __forceinline__ int32_t ld_relaxed_shared(const int32_t* p) {
   int32_t v;
   asm volatile("ld.relaxed.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
   return v;
+}
+__device__ __forceinline__ int32_t ld_acquire_shared(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_shared(int32_t* p, int32_t v) {
+  asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+// TMA bulk tensor store of one box of a 1-D int32 map: global rows
+// [x, x + box) <- shared rows at src (128-B aligned); rows past the map's
+// extent are not written.
+__device__ __forceinline__ void tma_store_1d(const CUtensorMap* map, int32_t x, const int32_t* src) {
+  asm volatile("cp.async.bulk.tensor.1d.global.shared::cta.bulk_group [%0, {%1}], [%2];" ::"l"(map), "r"(x),
+               "r"(smem_u32(src))
+               : "memory");
 }
 __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
   uint32_t v;
@@ -347,10 +392,10 @@ __device__ __forceinline__ void window_sums(const MoSmem<M>& S, const MoParams& 
 }
 
 template <int M, bool HAS_NE>
-__global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P) {
+__global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_constant__ MoParams P) {
   using C = Cfg<M>;
   using SM = MoSmem<M>;
-  constexpr int TILE = C::TILE, VEC = C::VEC, NPK = C::NPK, W = C::W, INSLOTS = C::INSLOTS;
+  constexpr int TILE = C::TILE, VEC = C::VEC, NPK = C::NPK, W = C::W, INSLOTS = C::INSLOTS, D1 = C::D1;
   constexpr int RING = SM::RING;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   SM& S = *reinterpret_cast<SM*>(smem_raw);
@@ -363,6 +408,10 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
     S.demand = -1;
     S.a_va = 0;
     S.w_done = 0;
+    S.chain_done = 0;
+    S.end_tile = 0x7fffffff;
+    S.lb_done = 0;
+    for (int o = 0; o < M; ++o) S.pfx[o] = 0;
     for (int s = 0; s < INSLOTS; ++s) {
       mbar_init(&S.full[s], 1);
       mbar_init(&S.empty[s], 1);
@@ -383,6 +432,13 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
   const int64_t ntiles = n > 0 ? (nv + TILE - 1) / TILE : 0;
   const uint64_t tag = S.epoch & TAG_MASK;
 
+  // Aux warps (producer, look-back, writers) first; with RA_MO_REGS the
+  // register file is rebalanced: compute warpgroups get more registers, the
+  // latency-bound aux warpgroups fewer (setmaxnreg, whole warpgroups).
+#if RA_MO_REGS
+  static_assert(NCW % 4 == 0 && (BLOCK / 32) % 4 == 0, "setmaxnreg works on whole warpgroups");
+  if (warp >= NCW) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(RA_MO_AUXREGS));
+#endif
   if (warp == PRWARP) {
     // ========================= producer: partition + load =====================
 #ifndef RA_MO_LATE_TICKET
@@ -415,95 +471,99 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
     return;
   }
 
-  if (warp == LBWARP) {
+  if (warp >= LBWARP && warp < LBWARP + NLB) {
     // ========================= look-back: tile offsets ========================
+    // NLB warps; warp r resolves the CTA's tiles k = r, r + NLB, ...: its
+    // window (the tiles strictly between tile k-1 and tile k of this CTA) is
+    // bulk-copied into the warp's own window slot once tile k+D1 is counted
+    // (its predecessors' words are then almost surely published) or at once
+    // on demand (the ring is full), and summed; the sums of consecutive tiles
+    // then chain through shared memory (pfx, chain_done): a few instructions.
+    // The windows of NLB tiles are in flight and summed in parallel.
+    const int r = warp - LBWARP;
     const uint32_t want = (uint32_t)((FLAG_A | (tag << TAG_SHIFT)) >> 32);
-    int64_t prefix[M];  // inclusive prefixes of this CTA's last placed tile
-#pragma unroll
-    for (int o = 0; o < M; ++o) prefix[o] = 0;
-    int64_t t_last = -1;  // tile index of the newest window issued
-    int m = 0x7fffffff;   // this CTA's tile count, once its end marker is counted
 #ifdef RA_MO_WATCHDOG
     long long t_wd = clock64();
 #endif
-    auto counted = [&](int x) {
-      if (x >= m) return true;
-      if (!__all_sync(0xffffffffu, mbar_test(&S.counted[x % K], (uint32_t)((x / K) & 1)))) return false;
-      if (S.tidx[x % K] < 0) m = x;
-      return true;
-    };
-    // Windows are issued in tile order, up to Q in flight: tile c's window
-    // (the tiles strictly between this CTA's previous tile and tile c) once
-    // tile c+D1 is counted — its predecessors' words are then almost surely
-    // published — or at once on demand (the ring is full); tile k is resolved
-    // as soon as its window has landed.  One L2 round trip per tile would
-    // otherwise bound the CTA at ~1.4 us per tile.
-    int c = 0;  // next window to issue
-    for (int k = 0;;) {  // k: next tile to resolve
-      bool busy = false;
-      while (c < k + Q && c < m && counted(c) && c < m) {
-        if (!(__all_sync(0xffffffffu, ld_relaxed_shared(&S.demand) >= c) || counted(c + D1))) break;
-        const int64_t tc = S.tidx[c % K];
-        if (lane == 0) {
-          issue_window(S, P, c % Q, t_last + 1, tc);
-          PROF_STAMP(S.t_issue[c % Q]);
-          PROF_LAT(21, S.t_count[c % K]);
+    for (int k = r;; k += NLB) {
+      // tile k counted, or k is past the CTA's end marker (end_tile < k: done)
+      bool past = false;
+      for (int spins = 0;; ++spins) {
+        if (__all_sync(0xffffffffu, mbar_test(&S.counted[k % K], (uint32_t)((k / K) & 1)))) break;
+        if (__all_sync(0xffffffffu, ld_acquire_shared(&S.end_tile) < k)) {
+          past = true;
+          break;
         }
-        t_last = tc;
-        ++c;
-        busy = true;
+        if (spins > 2) __nanosleep(32);
+#ifdef RA_MO_WATCHDOG
+        if (spins == 40000000 && lane == 0) {
+          printf("select_multi watchdog: block %d look-back %d counted k %d end %d\n", (int)blockIdx.x, r, k, S.end_tile);
+          __trap();
+        }
+#endif
       }
-      if (k == m) {  // end marker: tell the writers
-        if (lane == 0) mbar_arrive(&S.placed[k % K]);
+      if (past) break;
+      const int64_t tc = S.tidx[k % K];
+      if (tc < 0) {  // end marker (tile k == the CTA's tile count): tell the writers after every placement
+        if (lane == 0) {
+          while (ld_acquire_shared(&S.chain_done) != k) {}
+          mbar_arrive(&S.placed[k % K]);
+        }
         break;
       }
-      if (k < c && __all_sync(0xffffffffu, mbar_test(&S.winfull[k % Q], (uint32_t)((k / Q) & 1)))) {
-        const int q = k % Q;
-        int64_t ws[M];
-        if (lane == 0) PROF_LAT(20, S.t_issue[q]);
-        PROF_T0(t_ws);
-        window_sums<M>(S, P, q, lane, want, ws);
-        PROF_ADD(17, t_ws);
-        const int64_t tc = S.whi[q];
-        __syncwarp();
-        if (lane == 0) {
-#pragma unroll
-          for (int o = 0; o < M; ++o) {
-            const int64_t g = prefix[o] + ws[o];
-            S.goff[k % K][o] = g;
-            prefix[o] = g + S.cnt[k % K][o];
-          }
-          if (tc == ntiles - 1) {  // the last tile: every tile has published; totals, then the epoch
-#pragma unroll
-            for (int o = 0; o < M; ++o) *P.d_count[o] = prefix[o];
-            st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
-          }
-          PROF_LAT(18, S.t_count[k % K]);
-          PROF_STAMP(S.t_placed[k % K]);
-          mbar_arrive(&S.placed[k % K]);
-        } else {
-#pragma unroll
-          for (int o = 0; o < M; ++o) prefix[o] += ws[o] + S.cnt[k % K][o];
-        }
-        __syncwarp();
-        ++k;
-        continue;
+      int64_t tprev = -1;
+      if (k > 0) {
+        MWAIT(&S.counted[(k - 1) % K], (uint32_t)(((k - 1) / K) & 1), 2, k - 1);
+        tprev = S.tidx[(k - 1) % K];
       }
-#ifndef RA_MO_LBSLEEP
-#define RA_MO_LBSLEEP 64
-#endif
-      if (!busy && RA_MO_LBSLEEP > 0) __nanosleep(RA_MO_LBSLEEP);
+      // due: tile k+D1 counted (or the end marker), or the ring waits for tile k
+      for (int spins = 0;; ++spins) {
+        if (__all_sync(0xffffffffu, ld_relaxed_shared(&S.demand) >= k)) break;
+        if (__all_sync(0xffffffffu, mbar_test(&S.counted[(k + D1) % K], (uint32_t)(((k + D1) / K) & 1)))) break;
+        if (__all_sync(0xffffffffu, ld_acquire_shared(&S.end_tile) <= k + D1)) break;
+        if (spins > 2) __nanosleep(32);
 #ifdef RA_MO_WATCHDOG
-      if (!busy && clock64() - t_wd > 8000000000ll) {
-        if (lane == 0)
-          printf("select_multi watchdog: block %d look-back k %d c %d m %d demand %d\n", (int)blockIdx.x, k, c, m,
-                 S.demand);
-        __trap();
-      }
-      if (busy) t_wd = clock64();
+        if (spins == 40000000 && lane == 0) {
+          printf("select_multi watchdog: block %d look-back %d due k %d demand %d\n", (int)blockIdx.x, r, k, S.demand);
+          __trap();
+        }
 #endif
+      }
+      if (lane == 0) {
+        issue_window(S, P, r, tprev + 1, tc);
+        PROF_STAMP(S.t_issue[r]);
+        PROF_LAT(21, S.t_count[k % K]);
+      }
+      MWAIT(&S.winfull[r], (uint32_t)((k / NLB) & 1), 3, k);
+      if (lane == 0) PROF_LAT(20, S.t_issue[r]);
+      int64_t ws[M];
+      PROF_T0(t_ws);
+      window_sums<M>(S, P, r, lane, want, ws);
+      PROF_ADD(17, t_ws);
+      __syncwarp();
+      if (lane == 0) {
+        while (ld_acquire_shared(&S.chain_done) != k) {}  // tile k-1 placed: its prefix is in pfx
+#pragma unroll
+        for (int o = 0; o < M; ++o) {
+          const int64_t g = S.pfx[o] + ws[o];
+          S.goff[k % K][o] = g;
+          S.pfx[o] = g + S.cnt[k % K][o];
+        }
+        if (tc == ntiles - 1) {  // the last tile: every tile has published; totals, then the epoch
+#pragma unroll
+          for (int o = 0; o < M; ++o) *P.d_count[o] = S.pfx[o];
+          st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
+        }
+        PROF_LAT(18, S.t_count[k % K]);
+        PROF_STAMP(S.t_placed[k % K]);
+        st_release_shared(&S.chain_done, k + 1);
+        mbar_arrive(&S.placed[k % K]);
+      }
+      __syncwarp();
     }
-    if (lane == 0) {  // last CTA out: reset the ticket; at a tag wrap clear every status word
+    // the CTA's last look-back warp out joins the grid-wide epilogue:
+    // last CTA out resets the ticket; at a tag wrap it clears every status word
+    if (lane == 0 && atomicAdd(&S.lb_done, 1) == NLB - 1) {
       __threadfence();
       if (atomicAdd(&P.hdr[H_DONE], 1u) == gridDim.x - 1) {
         *P.ticket = 0ull;
@@ -524,44 +584,73 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
 
   if (warp >= WR0) {
     // ========================= writers: ring -> outputs =======================
+    // RA_MO_TMA: one elected lane streams each placed run with TMA bulk tensor
+    // stores (boxes of 256 and 32 rows at element coordinates) and the warp
+    // writes the last < 32 rows.  Default: NWR writer warps copy with
+    // coalesced 128-B warp stores, WU loads in flight per lane (measured
+    // faster on B200 for dense runs: DESIGN.md §7).  Plain stores also serve
+    // outputs that cannot take a TMA map (capacity >= 2^31 rows).
     const int wt = tid - 32 * WR0;
+    constexpr int WT = 32 * NWR, WU = RA_MO_WU;
     for (int k = 0;; ++k) {
       MWAIT(&S.placed[k % K], (uint32_t)((k / K) & 1), 4, (int)k);
       if (S.tidx[k % K] < 0) break;
       MWAIT(&S.scattered[k % K], (uint32_t)((k / K) & 1), 5, (int)k);
+      if (RA_MO_TMA && wt == 0) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // ring -> copy engine
+      if (RA_MO_TMA) __syncwarp();
       int32_t base = S.start[k % K];
       PROF_T0(t_wr);
 #pragma unroll
       for (int o = 0; o < M; ++o) {
         const int32_t c = S.cnt[k % K][o];
         const int64_t g = S.goff[k % K][o];
-        int64_t lim = P.out_cap[o] - g;
-        lim = lim < 0 ? 0 : (lim > c ? c : lim);
-        int32_t* __restrict__ out = P.out[o] + g;
         const int32_t* run = S.ring + base;
-        int e = wt;
-        for (; e + 3 * 32 * NWR < (int)lim; e += 4 * 32 * NWR) {
-          const int32_t a0 = run[e], a1 = run[e + 32 * NWR], a2 = run[e + 64 * NWR], a3 = run[e + 96 * NWR];
-          out[e] = a0;
-          out[e + 32 * NWR] = a1;
-          out[e + 64 * NWR] = a2;
-          out[e + 96 * NWR] = a3;
+        int32_t* __restrict__ out = P.out[o] + g;
+        const int64_t cap = P.out_cap[o] - g;  // rows of this run that fit
+        if (RA_MO_TMA && P.tma[o]) {
+          const int32_t i32 = c & ~31;
+          if (wt == 0 && g < P.out_cap[o]) {
+            const int32_t G = (int32_t)(g + P.omis[o]);
+            int32_t i = 0;
+            for (; i + 256 <= c; i += 256) tma_store_1d(&P.tmap[o][0], G + i, run + i);
+            for (; i < i32; i += 32) tma_store_1d(&P.tmap[o][1], G + i, run + i);
+          }
+          const int32_t e = i32 + wt;
+          if (wt < 32 && e < c && e < cap) out[e] = run[e];
+        } else {
+          const int64_t lim = cap < 0 ? 0 : (cap > c ? c : cap);
+          int e = wt;
+          for (; e + (WU - 1) * WT < (int)lim; e += WU * WT) {
+            int32_t a[WU];
+#pragma unroll
+            for (int u = 0; u < WU; ++u) a[u] = run[e + u * WT];
+#pragma unroll
+            for (int u = 0; u < WU; ++u) out[e + u * WT] = a[u];
+          }
+          for (; e < (int)lim; e += WT) out[e] = run[e];
         }
-        for (; e < (int)lim; e += 32 * NWR) out[e] = run[e];
-        base += c;
+        base += (c + 31) & ~31;
       }
-      writer_bar();  // every writer's ring reads are done
+      if (RA_MO_TMA && wt == 0) {
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the copy engine has read the runs
+      }
+      writer_bar();  // every writer is done reading the ring
       PROF_ADD(16, t_wr);
       if (wt == 0) {
         PROF_LAT(19, S.t_placed[k % K]);
         st_relaxed_shared(&S.w_done, k + 1);
-        mbar_arrive(&S.written[k % K]);  // release: the space and the counters above
+        mbar_arrive(&S.written[k % K]);  // release: the ring space
       }
     }
+    if (RA_MO_TMA && wt == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // outputs written
     return;
   }
 
   // ========================= compute groups =====================================
+#if RA_MO_REGS
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(RA_MO_REGS));
+#endif
   const int g = warp / GW, wg = warp % GW, gtid = tid - GT * g;
   for (int i = g;; i += NG) {
     const int slot = i % INSLOTS;
@@ -572,6 +661,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
       if (t == ntiles && gtid == 0) {  // the true end: tile i is this CTA's tile count
         if (i >= K) MWAIT(&S.written[i % K], (uint32_t)(((i / K) - 1) & 1), 7, (int)i);
         S.tidx[i % K] = -1;
+        st_release_shared(&S.end_tile, i);
         mbar_arrive(&S.counted[i % K]);
       }
       break;
@@ -633,11 +723,11 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
         const uint64_t a = (uint64_t)(uint32_t)agg[2 * j] | ((2 * j + 1 < M ? (uint64_t)(uint32_t)agg[2 * j + 1] : 0ull) << 16);
         dev::st_relaxed_u64(P.status + t * W + j, FLAG_A | (tag << TAG_SHIFT) | a);
       }
-      int32_t rows_in = 0;
+      int32_t rows_in = 0;  // the tile's runs, each padded to a multiple of 32 rows (128-B aligned starts)
 #pragma unroll
       for (int o = 0; o < M; ++o) {
         S.cnt[i % K][o] = agg[o];
-        rows_in += agg[o];
+        rows_in += (agg[o] + 31) & ~31;
       }
       S.tidx[i % K] = t;
       PROF_STAMP(S.t_count[i % K]);
@@ -706,7 +796,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const MoParams P
         for (int c = 0; c < 4; ++c) put_if(a, f, 1u << (4 * j + c), comp(v[j], c));
         r += (int32_t)((tot[q] >> (8 * b)) & 0xFFu);
       }
-      rb += agg[o];
+      rb += (agg[o] + 31) & ~31;
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&S.scattered[i % K]);
@@ -743,6 +833,30 @@ size_t mo_workspace_bytes(int64_t n) {
   return ((SEL_HDR_BYTES + 16 * (size_t)tiles + 16) + 255) / 256 * 256;
 }
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda)
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      f = nullptr;
+    return (PFN_cuTensorMapEncodeTiled_v12000)f;
+  }();
+  return fn;
+}
+
+// 1-D int32 map over out[0 .. cap) (from its 16-B aligned base, offset mis rows)
+bool encode_out_map(CUtensorMap* map, int32_t* out, int64_t cap, int32_t mis, uint32_t box) {
+  auto enc = tensor_map_encoder();
+  if (!enc) return false;
+  cuuint64_t dim[1] = {(cuuint64_t)(cap + mis)};
+  cuuint32_t boxd[1] = {box}, estr[1] = {1};
+  return enc(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 1, (void*)(out - mis), dim, nullptr, boxd, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int M, int32_t* const* d_outs,
                         const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s) {
   if (M < 1 || M > RA_MAX_OUTPUTS) return fail(RA_E_INVAL, "M=%d outside [1, %d]", M, RA_MAX_OUTPUTS);
@@ -772,6 +886,13 @@ int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int
     P.out[o] = d_outs[o];
     P.out_cap[o] = out_caps[o];
     P.d_count[o] = d_counts[o];
+    // TMA stores need element coordinates (int32) below 2^31: outputs whose
+    // rows (and the input's) stay below that; others take plain stores
+    P.omis[o] = (int32_t)(((uintptr_t)d_outs[o] & 15u) >> 2);
+    P.tma[o] = 0;
+    if (out_caps[o] > 0 && n + 64 < ((int64_t)1 << 31) && out_caps[o] + P.omis[o] < ((int64_t)1 << 31))
+      P.tma[o] = encode_out_map(&P.tmap[o][0], d_outs[o], out_caps[o], P.omis[o], 256) &&
+                 encode_out_map(&P.tmap[o][1], d_outs[o], out_caps[o], P.omis[o], 32);
   }
   const int64_t tile = mo_tile_rows(M);
   const int64_t ntiles = n > 0 ? (n + P.mis + tile - 1) / tile : 0;

@@ -192,6 +192,68 @@ def mixed_peak(w: float):
     return None
 
 
+def ncu_pcie(key: str):
+    """PCIe bytes (read = host->device) of one fission call from the committed
+    ncu application-range capture (scripts/pcie_ranges.py), if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_pcie.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f).get(key)
+    return None
+
+
+_PCIE = {}
+
+
+def pcie_peaks(torch):
+    """Pinned host<->device copy bandwidth measured here (the paper's Fig 4(b)
+    method): 1 GiB cudaMemcpyAsync each way, best of 3, CUDA events."""
+    if _PCIE:
+        return _PCIE
+    nb, ch = 1 << 30, 1 << 24
+    h = torch.empty(nb, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nb, dtype=torch.uint8, device="cuda")
+    cur = torch.cuda.current_stream()
+    st = [torch.cuda.Stream() for _ in range(3)]
+
+    def chunked(h2d):  # the fission pattern without kernels: 16 MiB chunks round-robin on 3 streams
+        for s_ in st:
+            s_.wait_stream(cur)
+        for c, o in enumerate(range(0, nb, ch)):
+            with torch.cuda.stream(st[c % 3]):
+                (d[o:o + ch].copy_(h[o:o + ch], non_blocking=True) if h2d else
+                 h[o:o + ch].copy_(d[o:o + ch], non_blocking=True))
+        for s_ in st:
+            cur.wait_stream(s_)
+
+    for name, fns in (("h2d_gbs", (lambda: d.copy_(h, non_blocking=True), lambda: chunked(True))),
+                      ("d2h_gbs", (lambda: h.copy_(d, non_blocking=True), lambda: chunked(False)))):
+        best = 0.0
+        for fn in fns:
+            for _ in range(3):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                fn()
+                e1.record()
+                e1.synchronize()
+                best = max(best, nb / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+        _PCIE[name] = best
+    _PCIE["how"] = ("pinned 1 GiB cudaMemcpyAsync, one copy or 16 MiB chunks on 3 streams, best of 3 each, "
+                    "measured in this run")
+    del h, d
+    return _PCIE
+
+
+def pcie_roofline(torch, h2d_bytes, seconds, ncu_key):
+    pk = pcie_peaks(torch)
+    ach = h2d_bytes / seconds / 1e9
+    cap = ncu_pcie(ncu_key)
+    return {"bound": "pcie", "achieved": ach, "peak": pk["h2d_gbs"], "unit": "GB/s", "frac": ach / pk["h2d_gbs"],
+            "peak_source": pk["how"], "d2h_peak": pk["d2h_gbs"],
+            "traffic": cap["pcie_read_bytes"] if cap else None,
+            "traffic_note": "ncu pcie__read_bytes.sum of one call (application-range replay), profiles/ncu_pcie.json"}
+
+
 def ncu_traffic(key: str):
     """dram bytes per launch from the committed ncu --set full capture, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -362,9 +424,9 @@ def run_ours(args, D: Dist):
                    "l2": "inputs > L2 (1 GiB column per step vs 126 MB L2), no flush needed",
                    "parallelism": f"row-range shards x{D.world}, NCCL all_gather of counts"},
         "gpu_launches": launches,
-        "roofline": {"kernel": "select_fused_kernel", "bound": "hbm", "achieved": achieved, "peak": peak,
-                     "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": ncu_traffic(f"select_fused_k{k}_s{s_sel}_n{args.rows_log2}"),
+        "roofline": {"kernel": "select_multi_kernel<M=1> (the fused chain)", "bound": "hbm", "achieved": achieved,
+                     "peak": peak, "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": ncu_traffic(f"select_chain_k{k}_s{s_sel}_n{args.rows_log2}"),
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kms,
                      "mixed_stream_peak": mixed_peak(kept / n),
                      "frac_of_mixed_stream_peak": (achieved / mixed_peak(kept / n)) if mixed_peak(kept / n) else None},
@@ -423,7 +485,8 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
         ex["e2e"] = {"value": D.world * n / dt, "unit": "rows/s", "h2d_bytes_per_step": 4 * n,
                      "d2h_bytes_per_step": 4 * c + 8 * ((n + chunk - 1) // chunk), "ms_per_step": dt * 1e3,
                      "path": "ra_fission_run: pinned host in/out, chunk 2^24 rows, 3 streams (fusion+fission)",
-                     "pcie_h2d_gbs": 4 * n / dt / 1e9}
+                     "pcie_h2d_gbs": 4 * n / dt / 1e9,
+                     "roofline": pcie_roofline(torch, 4 * n, dt, "select_fission_n28")}
         # d4: the paper's Fig 16 modes on the same host-resident chain
         modes = {"serial": (n, 1, False), "fusion_only": (n, 1, True),
                  "fission_only": (chunk, 3, False), "fusion_fission": (chunk, 3, True)}
@@ -475,7 +538,8 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                             "rows": n3, "kept": k3, "ms_per_step": f3ms, "rows_per_s": n3 / (f3ms * 1e-3),
                             "checked": "count + 65536 sampled outputs equal the device-resident fused chain",
                             "h2d_bytes_per_step": 4 * n3, "d2h_bytes_per_step": 4 * k3 + 8 * (n3 >> 24),
-                            "pcie_h2d_gbs": 4 * n3 / (f3ms * 1e-3) / 1e9}
+                            "pcie_h2d_gbs": 4 * n3 / (f3ms * 1e-3) / 1e9,
+                            "roofline": pcie_roofline(torch, 4 * n3, f3ms * 1e-3, "select_fission_n30")}
         del h3, o3
 
     # --- d5 shape for SELECT: 2^30 device-resident rows split across the ranks
@@ -504,44 +568,55 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                                           f"s={s_sel}/stage (SURVEY d5 shape)",
                               "rows": 1 << 30, "rows_per_s": (1 << 30) / (bms * 1e-3), "ms_per_step": bms,
                               "kernel_ms": bkms, "scaling": "strong",
-                              "roofline": {"kernel": "select_fused_kernel", "bound": "hbm", "achieved": bach,
+                              "roofline": {"kernel": "select_multi_kernel<M=1>", "bound": "hbm", "achieved": bach,
                                            "peak": peak, "unit": "GB/s", "frac": bach / peak}}
     del xb, ob, wsb
 
-    # --- f2: two SELECTs filtering the same input (Fig 2(c)): one fused pass
-    # vs the two SELECT kernels run one after the other (two input reads)
-    chains = [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)]]
-    mo = [torch.empty(n, dtype=torch.int32, device=dev) for _ in range(2)]
-    mc = torch.zeros(2, dtype=torch.int64, device=dev)
-    mws_b = R.ra_select_multi_workspace_bytes(n)
-    mws = torch.zeros(mws_b, dtype=torch.uint8, device=dev)
-    keepP = [R.make_preds(c) for c in chains]
-    mch = (ctypes.c_void_p * 2)(*[ctypes.addressof(p_) for p_ in keepP])
-    mks = (ctypes.c_int * 2)(*[len(c) for c in chains])
-    mop = (ctypes.c_void_p * 2)(*[o.data_ptr() for o in mo])
-    mcap = (ctypes.c_int64 * 2)(n, n)
-    mcp = (ctypes.c_void_p * 2)(mc.data_ptr(), mc.data_ptr() + 8)
-    am = (x.data_ptr(), n, mch, mks, 2, mop, mcap, mcp, mws.data_ptr(), mws_b, sh)
-    mms, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_multi(*am), 20, 3)
-    c0, c1 = (int(v) for v in mc.cpu().tolist())
-    sep = [(x.data_ptr(), n, keepP[o], len(chains[o]), 1, mo[o].data_ptr(), n, mc.data_ptr() + 8 * o,
-            mws.data_ptr(), mws_b, sh) for o in range(2)]
+    # --- f2: several SELECTs filtering the same input (Fig 2(c)): one fused pass
+    # (select_multi_kernel<M>, one input read) vs the M SELECT passes run one
+    # after the other (M input reads); M = 2 (the bench pair) and M = 4
+    def multi_leg(chains, key):
+        M = len(chains)
+        mo = [torch.empty(n, dtype=torch.int32, device=dev) for _ in range(M)]
+        mc = torch.zeros(M, dtype=torch.int64, device=dev)
+        mws_b = R.ra_select_multi_workspace_bytes(n)
+        mws = torch.zeros(mws_b, dtype=torch.uint8, device=dev)
+        keepP = [R.make_preds(c) for c in chains]
+        mch = (ctypes.c_void_p * M)(*[ctypes.addressof(p_) for p_ in keepP])
+        mks = (ctypes.c_int * M)(*[len(c) for c in chains])
+        mop = (ctypes.c_void_p * M)(*[o.data_ptr() for o in mo])
+        mcap = (ctypes.c_int64 * M)(*([n] * M))
+        mcp = (ctypes.c_void_p * M)(*[mc.data_ptr() + 8 * o for o in range(M)])
+        am = (x.data_ptr(), n, mch, mks, M, mop, mcap, mcp, mws.data_ptr(), mws_b, sh)
+        mms, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_multi(*am), 20, 3)
+        cs = [int(v) for v in mc.cpu().tolist()]
+        sws_b = R.ra_select_workspace_bytes(n, RA_MAX_PREDS, 1)
+        sws = torch.zeros(sws_b, dtype=torch.uint8, device=dev)
+        sep = [(x.data_ptr(), n, keepP[o], len(chains[o]), 1, mo[o].data_ptr(), n, mc.data_ptr() + 8 * o,
+                sws.data_ptr(), sws_b, sh) for o in range(M)]
 
-    def two_kernels(i=0, kernel_done=False):
-        R.ra_select_chain(*sep[0])
-        R.ra_select_chain(*sep[1])
-    sms, _ = timed(torch, D, two_kernels, 20, 3)
-    assert [int(v) for v in mc.cpu().tolist()] == [c0, c1]
-    malg = 4 * n + 4 * (c0 + c1)
-    mach = malg / (mms * 1e-3) / 1e9
-    ex["select_multi"] = {"outputs": 2, "chains": [[list(p_) for p_ in c] for c in chains], "kept": [c0, c1],
-                          "rows_per_s": D.world * n / (mms * 1e-3), "ms_per_step": mms,
-                          "two_separate_selects_ms": sms, "fused_over_separate": sms / mms,
-                          "bytes_ratio": (8 * n + 4 * (c0 + c1)) / malg,
-                          "roofline": {"kernel": "select_fused_kernel<M=2>", "bound": "hbm", "achieved": mach,
-                                       "peak": peak, "unit": "GB/s", "frac": mach / peak,
-                                       "algorithmic_bytes_per_launch": malg}}
-    del mo, mws
+        def separate(i=0, kernel_done=False):
+            for a in sep:
+                R.ra_select_chain(*a)
+        sms, _ = timed(torch, D, separate, 20, 3)
+        assert [int(v) for v in mc.cpu().tolist()] == cs
+        malg = 4 * n + 4 * sum(cs)
+        mach = malg / (mms * 1e-3) / 1e9
+        return {"outputs": M, "chains": [[list(p_) for p_ in c] for c in chains], "kept": cs,
+                "rows_per_s": D.world * n / (mms * 1e-3), "ms_per_step": mms,
+                "separate_selects_ms": sms, "fused_over_separate": sms / mms,
+                "bytes_ratio": (4 * M * n + 4 * sum(cs)) / malg,
+                "roofline": {"kernel": f"select_multi_kernel<M={M}>", "bound": "hbm", "achieved": mach,
+                             "peak": peak, "unit": "GB/s", "frac": mach / peak, "algorithmic_bytes_per_launch": malg,
+                             "traffic": ncu_traffic(key),
+                             "mixed_stream_peak": mixed_peak(sum(cs) / n),
+                             "frac_of_mixed_stream_peak": mach / mixed_peak(sum(cs) / n) if mixed_peak(sum(cs) / n)
+                             else None}}
+
+    from paper_conf_ipps_wudwcyc12_b200 import RA_MAX_PREDS
+    ex["select_multi"] = multi_leg([[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)]], "select_multi_m2_s0.5_n28")
+    ex["select_multi"]["m4"] = multi_leg([[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)], [("ge", 2**30)],
+                                          [("lt", -(2**30))]], "select_multi_m4_n28")
 
     # --- f3: tuple SELECT (Table I) on the same key column + two int32 fields,
     # the same chain; outputs the key and both fields of the selected rows
@@ -703,6 +778,7 @@ def q1_e2e(args, D, torch, R, sf):
     res = {"value": N / (ms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 38 * N,
            "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": ms,
            "pcie_h2d_gbs": 38 * N / (ms * 1e-3) / 1e9, "groups": len(rows), "finalize_rc": rc,
+           "roofline": pcie_roofline(torch, 38 * N, ms * 1e-3, "q1_fission_sf10"),
            "path": "ra_q1_fission_run: pinned host columns, chunk 2^22 rows, 3 streams"}
     # f1 x f4: the same table held narrow (11 B/row) in pinned host memory
     dcols = {k: v.cuda() for k, v in h.items()}
@@ -724,6 +800,7 @@ def q1_e2e(args, D, torch, R, sf):
     res["narrow"] = {"value": N / (nms * 1e-3), "unit": "rows/s", "h2d_bytes_per_step": 11 * N,
                      "d2h_bytes_per_step": 3 * ctypes.sizeof(R.ra_q1_partial), "ms_per_step": nms,
                      "pcie_h2d_gbs": 11 * N / (nms * 1e-3) / 1e9,
+                     "roofline": pcie_roofline(torch, 11 * N, nms * 1e-3, "q1n_fission_sf10"),
                      "path": "ra_q1_narrow_fission_run: pinned host narrow columns, chunk 2^23 rows, 3 streams"}
     del hn
     return res

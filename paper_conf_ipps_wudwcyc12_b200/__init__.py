@@ -76,6 +76,9 @@ def workspace(device, kind: str, nbytes: int, stream=None):
     key = (str(device), kind, _stream_handle(stream))
     ws = _WS.get(key)
     if ws is None or ws.numel() < nbytes:
+        if torch.cuda.is_current_stream_capturing():
+            raise RuntimeError(f"workspace {kind!r} for this stream must be created before CUDA-graph capture "
+                               "(make one call on the capture stream first)")
         ws = torch.zeros(max(256, nbytes), dtype=torch.uint8, device=device)
         # Root cause of round 1's one-off Q1-fission mismatch: without this the
         # fill kernel (current stream) could still be running while the fission

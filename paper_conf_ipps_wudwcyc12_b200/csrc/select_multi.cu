@@ -36,6 +36,7 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "ra_internal.cuh"
@@ -114,12 +115,14 @@ __host__ __device__ constexpr int q_of(int npk, int j) { return npk == 2 ? (j & 
 __host__ __device__ constexpr int b_of(int npk, int j) { return npk == 2 ? (j >> 1) : ((j >> 1) | ((j & 1) << 1)); }
 
 struct MoParams {
+#if RA_MO_TMA
   // per output: 1-D TMA maps of the output (int32, element coordinates from
   // its 16-B aligned base, bounded by out_cap: the copy engine clips rows past
   // the capacity) with boxes of 256 and 32 rows; tma[o] = 0: plain stores
   CUtensorMap tmap[RA_MAX_OUTPUTS][2];
-  int32_t tma[RA_MAX_OUTPUTS];
   int32_t omis[RA_MAX_OUTPUTS];  // rows of out[o]'s 16-B chunk before out[o]
+#endif
+  int32_t tma[RA_MAX_OUTPUTS];
   const int32_t* abase;  // 16-B aligned base, = d_in - mis
   int64_t n;
   uint32_t* hdr;
@@ -607,7 +610,8 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
         const int32_t* run = S.ring + base;
         int32_t* __restrict__ out = P.out[o] + g;
         const int64_t cap = P.out_cap[o] - g;  // rows of this run that fit
-        if (RA_MO_TMA && P.tma[o]) {
+#if RA_MO_TMA
+        if (P.tma[o]) {
           const int32_t i32 = c & ~31;
           if (wt == 0 && g < P.out_cap[o]) {
             const int32_t G = (int32_t)(g + P.omis[o]);
@@ -617,7 +621,9 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
           }
           const int32_t e = i32 + wt;
           if (wt < 32 && e < c && e < cap) out[e] = run[e];
-        } else {
+        } else
+#endif
+        {
           const int64_t lim = cap < 0 ? 0 : (cap > c ? c : cap);
           int e = wt;
           for (; e + (WU - 1) * WT < (int)lim; e += WU * WT) {
@@ -815,6 +821,10 @@ int launch_mo(const MoParams& P, int64_t ntiles, cudaStream_t s) {
   });
   if (a < 0) return a;
   int64_t grid = num_sms();  // persistent: one CTA per SM
+  // RA_SEL_MAX_CTAS (diagnostics only): cap the grid, for the paper's Fig 12
+  // experiment (a SELECT with half the CTAs, two of them on two streams)
+  static const int64_t max_ctas = getenv("RA_SEL_MAX_CTAS") ? atoll(getenv("RA_SEL_MAX_CTAS")) : 0;
+  if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
   if (grid > ntiles) grid = ntiles;
   if (grid < 1) grid = 1;
   cudaError_t e = launch_pdl(select_multi_kernel<M, HAS_NE>, dim3((unsigned)grid), dim3(BLOCK), sizeof(MoSmem<M>), s, P);
@@ -833,6 +843,7 @@ size_t mo_workspace_bytes(int64_t n) {
   return ((SEL_HDR_BYTES + 16 * (size_t)tiles + 16) + 255) / 256 * 256;
 }
 
+#if RA_MO_TMA
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda)
 PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
@@ -856,6 +867,7 @@ bool encode_out_map(CUtensorMap* map, int32_t* out, int64_t cap, int32_t mis, ui
              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
+#endif
 
 int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int M, int32_t* const* d_outs,
                         const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s) {
@@ -888,11 +900,13 @@ int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int
     P.d_count[o] = d_counts[o];
     // TMA stores need element coordinates (int32) below 2^31: outputs whose
     // rows (and the input's) stay below that; others take plain stores
-    P.omis[o] = (int32_t)(((uintptr_t)d_outs[o] & 15u) >> 2);
     P.tma[o] = 0;
+#if RA_MO_TMA
+    P.omis[o] = (int32_t)(((uintptr_t)d_outs[o] & 15u) >> 2);
     if (out_caps[o] > 0 && n + 64 < ((int64_t)1 << 31) && out_caps[o] + P.omis[o] < ((int64_t)1 << 31))
       P.tma[o] = encode_out_map(&P.tmap[o][0], d_outs[o], out_caps[o], P.omis[o], 256) &&
                  encode_out_map(&P.tmap[o][1], d_outs[o], out_caps[o], P.omis[o], 32);
+#endif
   }
   const int64_t tile = mo_tile_rows(M);
   const int64_t ntiles = n > 0 ? (n + P.mis + tile - 1) / tile : 0;

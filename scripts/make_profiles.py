@@ -18,10 +18,14 @@ OUT = os.path.join(ROOT, "profiles")
 os.makedirs(OUT, exist_ok=True)
 
 CAPTURES = {  # report -> (summary name, traffic key, command)
-    "prof_select": ("select_k2_s05_n28", "select_fused_k2_s0.5_n28",
-                    "python scripts/prof_driver.py select 5  (2^28 int32, k=2, s=0.5/stage)"),
-    "prof_select_s01": ("select_k1_s001_n28", "select_fused_k1_s0.01_n28",
-                        "python scripts/prof_driver.py select 5 28 1 0.01  (2^28 int32, k=1, s=0.01)"),
+    "prof_select": ("select_chain_k2_s05_n28", "select_chain_k2_s0.5_n28",
+                    "python scripts/prof_driver.py select 5  (2^28 int32, k=2, s=0.5/stage; select_multi_kernel<1>)"),
+    "prof_select_s01": ("select_chain_k1_s001_n28", "select_chain_k1_s0.01_n28",
+                        "python scripts/prof_driver.py select 5 28 1 0.01  (2^28 int32, k=1, s=0.01; select_multi_kernel<1>)"),
+    "prof_select_s09": ("select_chain_k1_s09_n28", "select_chain_k1_s0.9_n28",
+                        "python scripts/prof_driver.py select 5 28 1 0.9  (2^28 int32, k=1, s=0.9; select_multi_kernel<1>)"),
+    "prof_unfused": ("unfused_pass_k2_s05_n28", "unfused_pass_k2_s0.5_n28",
+                     "python scripts/prof_driver.py unfused 5  (first pass of the unfused chain: select_fused_kernel)"),
     "prof_q1": ("q1_sf10", "q1_sf10", "python scripts/prof_driver.py q1 5  (SF10, 60M rows)"),
     "prof_rows": ("select_rows_k2_s05_n28", "select_rows_k2_s0.5_n28",
                   "python scripts/prof_driver.py rows 5  (2^28 key + 2 int32 fields, k=2, s=0.5/stage)"),
@@ -114,7 +118,7 @@ if os.path.exists(ppath):
     for r in rows[1:]:
         per.setdefault(int(r[ii]), {})[r[mi]] = (r[vi], r[ui])
     pcie = {}
-    lines = [f"# round {RND}: ncu --replay-mode app-range --profile-from-start off --metrics "
+    lines = [f"# round {RND}: ncu --replay-mode app-range --metrics "
              "pcie__read_bytes.sum,pcie__write_bytes.sum,gpu__time_duration.sum python scripts/pcie_ranges.py",
              "# one range = one synchronous fission call (H2D + kernels + D2H); read = host->device over PCIe",
              "# range                    pcie_read_bytes   pcie_write_bytes   range_ms   read GB/s"]

@@ -101,14 +101,18 @@ constexpr int WIN_WORDS = 512;                // window slot (status words)
 constexpr int SMEM_BUDGET = 232448;           // max dynamic shared memory per CTA on sm_100
 
 
+#ifndef RA_MO_VEC34
+#define RA_MO_VEC34 8     // M = 3, 4: int4 vectors per compute lane per tile
+#define RA_MO_IN_KB34 64  //           input ring per CTA
+#endif
 template <int M>
 struct Cfg {
-  static constexpr int VEC = M <= 2 ? 8 : 4;        // int4 vectors per compute lane per tile
+  static constexpr int VEC = M <= 2 ? 8 : RA_MO_VEC34;  // int4 vectors per compute lane per tile
   static constexpr int TILE = GT * VEC * 4;          // rows per tile: 8192 | 4096
   static constexpr int WROWS = TILE / GW;            // contiguous rows per compute warp
   static constexpr int NPK = VEC / 4;                // packed 8-bit count words per lane per output
   static constexpr int W = (M + 1) / 2;              // status words per tile
-  static constexpr int INSLOTS = RA_MO_IN_KB * 1024 / (TILE * 4);
+  static constexpr int INSLOTS = (M <= 2 ? RA_MO_IN_KB : RA_MO_IN_KB34) * 1024 / (TILE * 4);
   static constexpr int D1 = RA_MO_D1 > 0 ? RA_MO_D1 : (M == 1 ? 2 : 1);
 };
 __host__ __device__ constexpr int q_of(int npk, int j) { return npk == 2 ? (j & 1) : 0; }
@@ -175,8 +179,8 @@ struct __align__(128) MoSmem : MoFixed<M> {
   static constexpr int RING = ring_ints<M>();
   alignas(128) int32_t ring[RING];  // runs start at multiples of 32 rows (128 B): TMA store sources
 };
-static_assert(MoSmem<1>::RING >= 8192 && MoSmem<2>::RING >= 2 * 8192 && MoSmem<3>::RING >= 3 * 4096 &&
-                  MoSmem<4>::RING >= 4 * 4096,
+static_assert(MoSmem<1>::RING >= Cfg<1>::TILE && MoSmem<2>::RING >= 2 * Cfg<2>::TILE &&
+                  MoSmem<3>::RING >= 3 * Cfg<3>::TILE && MoSmem<4>::RING >= 4 * Cfg<4>::TILE,
               "a tile's M runs must always fit an empty ring");
 static_assert(sizeof(MoSmem<1>) <= SMEM_BUDGET && sizeof(MoSmem<2>) <= SMEM_BUDGET &&
                   sizeof(MoSmem<3>) <= SMEM_BUDGET && sizeof(MoSmem<4>) <= SMEM_BUDGET,
@@ -836,10 +840,12 @@ int launch_mo(const MoParams& P, int64_t ntiles, cudaStream_t s) {
 }  // namespace
 
 int64_t mo_tile_rows(int M) { return M <= 2 ? Cfg<1>::TILE : Cfg<3>::TILE; }
+static_assert(Cfg<3>::TILE == Cfg<4>::TILE, "one tile size for M = 3, 4");
 
 size_t mo_workspace_bytes(int64_t n) {
-  // worst case over M: 4096-row tiles (+3 rows of misalignment, +1), two words each
-  const int64_t tiles = (n + 3 + Cfg<3>::TILE - 1) / Cfg<3>::TILE + 1;
+  // worst case over M: the smaller tile (+3 rows of misalignment, +1), two words each
+  constexpr int64_t T = Cfg<1>::TILE < Cfg<3>::TILE ? Cfg<1>::TILE : Cfg<3>::TILE;
+  const int64_t tiles = (n + 3 + T - 1) / T + 1;
   return ((SEL_HDR_BYTES + 16 * (size_t)tiles + 16) + 255) / 256 * 256;
 }
 

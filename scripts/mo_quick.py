@@ -14,7 +14,7 @@ x = torch.empty(n, dtype=torch.int32, device="cuda")
 ragen.int32_column_dev(2, x)
 outs = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
 res = []
-for M, s in [(1, 0.01), (1, 0.25), (1, 0.5), (1, 0.9), (2, 0.5), (2, 0.9), (3, 0.01), (4, 0.5)]:
+for M, s in [(1, 0.01), (1, 0.25), (1, 0.5), (1, 0.9), (2, 0.5), (2, 0.9), (3, 0.01), (3, 0.5), (4, 0.01), (4, 0.5), (4, 0.9)]:
     ch = [[("lt", ragen.nested_thresholds(s, 1)[0])]] * M
     for _ in range(3):
         R.select_multi(x, ch, outs=outs[:M])

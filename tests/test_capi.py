@@ -41,9 +41,9 @@ def test_workspace_sizes():
     assert R.ra_select_workspace_bytes(1 << 28, 1, 0) == f  # k=1 never materialises
     assert R.ra_fission_workspace_bytes(1 << 20, 3, 2, 1) >= 3 * 2 * 4 * (1 << 20)
     assert R.ra_fission_workspace_bytes(0, 3, 2, 1) == 0
-    # several outputs: status words only, two per 4096-row tile at most (M = 3, 4)
+    # several outputs: status words only, two per 8192-row tile at most (M = 3, 4)
     m = R.ra_select_multi_workspace_bytes(1 << 28)
-    assert 16 * ((1 << 28) // 4096) <= m <= 16 * ((1 << 28) // 4096 + 2) + 512
+    assert 16 * ((1 << 28) // 8192) <= m <= 16 * ((1 << 28) // 8192 + 2) + 512
     assert R.ra_select_multi_workspace_bytes(1 << 10) < R.ra_select_multi_workspace_bytes(1 << 20) <= m
     # tuple SELECT: status words + order masks (n/8 + n/170 B) + id staging (4 B/row)
     t = R.ra_select_rows_workspace_bytes(1 << 28, 2)

@@ -290,7 +290,7 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   const bool masks = m > 0 && g.sparse_den > 0;
   const bool stage = !d_rowids && !masks;  // A/B: ids staged by the key pass
   rc = launch_select_pass(d_key, n, nullptr, cp, nullptr, cap, d_count, d_ws, (cudaStream_t)stream,
-                          (d_rowids && cap > 0) || stage ? ids : nullptr, nullptr, masks ? &mk : nullptr);
+                          (d_rowids && cap > 0) || stage ? ids : nullptr, masks ? &mk : nullptr);
   if (rc) return rc;
   if (masks && !d_rowids) {
     rc = ra::launch_ids_from_masks(d_key, n, mk, d_count, g.sparse_den, ids, (cudaStream_t)stream);

@@ -99,20 +99,11 @@ int64_t sel_max_tiles(int64_t n);  // tiles for n rows with any 16-B misalignmen
 size_t sel_status_bytes(int64_t n);
 size_t sel_inter_bytes(int64_t n);
 
-// One select pass (one kernel).  n_max = host bound on rows; d_n (nullable) =
-// device-resident actual row count (<= n_max) produced by a previous pass.
-// rows != nullptr: row-id mode (the selected rows' ids go to rows[0..out_cap),
-// d_out unused).
-// second != nullptr: a second predicate / output in the same pass (ra_select_multi).
-struct SelSecond {
-  CanonPred cp;
-  int32_t* out;
-  int64_t out_cap;
-  int64_t* d_count;
-  int32_t* spill;  // sel_spill_bytes(n) of workspace (second runs the ring cannot hold)
-};
-constexpr int SEL_MULTI_MAX_GRID = 320;  // CTAs of a two-output pass (>= 2 per SM on 148 SMs)
-size_t sel_spill_bytes(int64_t n);
+// One single-output select pass (select_fused_kernel: the unfused chain's
+// passes and the tuple SELECT's key pass).  n_max = host bound on rows; d_n
+// (nullable) = device-resident actual row count (<= n_max) produced by a
+// previous pass.  rows != nullptr: row-id mode (the selected rows' ids go to
+// rows[0..out_cap), d_out unused).
 // Row-id mode extras for the payload compaction (compact.cu), per select tile t
 // (SEL_TILE rows counted from the key's 16-B aligned base): the compute lanes'
 // flag words fmask[t*SEL_THREADS + tid] and a 48-B record meta[t*12 ..]: the
@@ -126,8 +117,7 @@ size_t sel_masks_bytes(int64_t n);
 
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, uint32_t* rows = nullptr, const SelSecond* second = nullptr,
-                       const SelMasks* masks = nullptr);
+                       cudaStream_t s, uint32_t* rows = nullptr, const SelMasks* masks = nullptr);
 
 // Several SELECTs on one input in one pass (select_multi.cu), 1 <= M <= 4:
 // cp[o] = output o's folded chain; validated arguments.

@@ -1,4 +1,9 @@
-// select_fused.cu — single-pass fused SELECT (chain) for sm_100a.
+// select_fused.cu — single-pass, single-output SELECT for sm_100a: the
+// passes of the unfused chain ("without round trip", one predicate per pass,
+// row count from the previous pass on the device) and the tuple SELECT's key
+// pass (row ids + order masks for the payload compaction).  The fused chain
+// and several SELECTs on one input run select_multi.cu's warp-specialised
+// pass (writer warps, cooperative look-back), measured faster on B200.
 //
 // The paper's SELECT has four stages — partition, filter, buffer, gather —
 // in two CUDA kernels separated by a global synchronisation so that each CTA
@@ -108,9 +113,6 @@ constexpr int K = LAG + 2;               // metadata slots: tiles counted but no
 #ifndef RA_SEL_PTXSCATTER
 #define RA_SEL_PTXSCATTER 1
 #endif
-#ifndef RA_SEL_SPILL_AT
-#define RA_SEL_SPILL_AT RING  // M == 2: a tile whose two runs exceed this spills its second run
-#endif
 #ifndef RA_SEL_BATCH
 #define RA_SEL_BATCH 1  // tiles per ticket (see the producer warp)
 #endif
@@ -138,7 +140,7 @@ __host__ __device__ constexpr int q_of(int j) { return NPK == 2 ? (j & 1) : 0; }
 __host__ __device__ constexpr int b_of(int j) { return NPK == 2 ? (j >> 1) : ((j >> 1) | ((j & 1) << 1)); }
 static_assert(NW <= 32, "one warp reduces the per-warp counts");
 static_assert(LAG >= D2 + 1, "a tile is placed before it is due");
-static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");  // (M == 2: 2 x SEL_TILE, SelSmem2)
+static_assert(SEL_OUTRING >= SEL_TILE, "a whole tile must fit the ring");
 
 struct SelParams {
   const int32_t* abase;  // 16-B aligned base, = d_in - mis
@@ -156,15 +158,6 @@ struct SelParams {
   // fmask[t][256] and meta[t][12] = the warps' exclusive bases + the tile offset
   uint32_t* fmask;
   uint32_t* meta;
-  // M == 2 (ra_select_multi): a second predicate and output on the same input
-  int32_t lo2;
-  uint32_t span2;
-  int32_t n_ne2;
-  int32_t ne2[RA_MAX_PREDS];
-  int32_t* out2;
-  int32_t* spill;  // M == 2: per-CTA global slots [K][SEL_TILE] for second runs the ring cannot hold
-  int64_t out_cap2;
-  int64_t* d_count2;
   int32_t lo;
   uint32_t span;  // hi - lo (the interval is never empty: see launch_select_pass)
   int32_t n_ne;
@@ -186,22 +179,15 @@ struct __align__(128) SelSmemT {
   int64_t tidx[K];                     // tile index of CTA-local tile k (-1: no more tiles)
   int64_t wlo[Q], whi[Q];              // window bounds [lo, hi) of each window slot
   int64_t goff[K];                     // tile output offsets
-  uint32_t wtot[2][2][NW];             // [tile parity][output][warp] selected counts
+  uint32_t wtot[2][NW];                // [tile parity][warp] selected counts
   int32_t cnt[K];                      // tile aggregates
-  int32_t cnt2[K];                     // M == 2: second output's tile aggregates (run after the first)
-  int64_t goff2[K];                    // M == 2: second output's tile offsets
   int32_t start[K];                    // tile run start in the ring
-  int32_t spilled[K];                  // M == 2: the tile's second run is in its spill slot
   int64_t n;
   uint32_t epoch;
   int32_t demand;  // oldest tile the compute warps are waiting to write (-1: none yet)
 };
-// A 40 KB ring (2 CTAs/SM), also for two outputs (ra_select_multi): a tile
-// whose two runs exceed it is placed straight from registers (the compute
-// loop's "direct" path).
+// A 40 KB ring (2 CTAs/SM).
 using SelSmem = SelSmemT<SEL_OUTRING>;
-template <int M>
-using SmemFor = SelSmem;
 
 using dev::smem_u32;
 using dev::mbar_init;
@@ -245,35 +231,11 @@ __device__ __forceinline__ bool keep(int32_t x, const SelParams& P) {
   return k;
 }
 
-template <bool HAS_NE>
-__device__ __forceinline__ bool keep2(int32_t x, const SelParams& P) {
-  bool k = (uint32_t)x - (uint32_t)P.lo2 <= P.span2;
-  if (HAS_NE) {
-#pragma unroll
-    for (int j = 0; j < RA_MAX_PREDS; ++j)
-      if (j < P.n_ne2) k &= (x != P.ne2[j]);
-  }
-  return k;
-}
-
 __device__ __forceinline__ int32_t comp(const int4& v, int c) {
   return c == 0 ? v.x : c == 1 ? v.y : c == 2 ? v.z : v.w;
 }
 
 // Store v at shared byte address a and advance a, iff (fl & mask) != 0.
-// The same into global memory (M == 2 spill slots).
-__device__ __forceinline__ void put_if_global(int32_t*& a, uint32_t fl, uint32_t mask, int32_t v) {
-  asm volatile(
-      "{\n\t.reg .pred q;\n\t.reg .b32 t;\n\t"
-      "and.b32 t, %1, %2;\n\t"
-      "setp.ne.u32 q, t, 0;\n\t"
-      "@q st.global.b32 [%0], %3;\n\t"
-      "@q add.u64 %0, %0, 4;\n\t}"
-      : "+l"(a)
-      : "r"(fl), "r"(mask), "r"(v)
-      : "memory");
-}
-
 __device__ __forceinline__ void put_if(uint32_t& a, uint32_t fl, uint32_t mask, int32_t v) {
   asm volatile(
       "{\n\t.reg .pred q;\n\t.reg .b32 t;\n\t"
@@ -367,57 +329,9 @@ __device__ __forceinline__ int64_t window_sum(const SM& S, const SelParams& P, i
   return total;
 }
 
-// M == 2: the status word carries both outputs' aggregates (16 bits each in
-// the low word); sum them separately.  Same readiness rule as window_sum.
-template <typename SM>
-__device__ __forceinline__ void window_sum2(const SM& S, const SelParams& P, int q, int lane, uint32_t want,
-                                            int64_t& t0, int64_t& t1) {
-  const int64_t lo = S.wlo[q], hi = S.whi[q];
-  const int64_t s0 = lo & ~1ll;
-  const bool copied = hi > lo && hi - s0 <= WIN_WORDS;
-  const uint64_t pad = (uint64_t)want << 32;
-  t0 = t1 = 0;
-  for (int64_t base = lo; base < hi; base += PASS_WORDS) {
-    uint64_t w[LBW];
-    if (copied) {
-#pragma unroll
-      for (int c = 0; c < LBW; ++c) {
-        const int64_t idx = base + lane + 32 * c;
-        const bool in = idx < hi;
-        const uint64_t x = S.win[q][(in ? idx : lo) - s0];
-        w[c] = in ? x : pad;
-      }
-    } else {
-#pragma unroll
-      for (int c = 0; c < LBW; ++c) {
-        const int64_t idx = base + lane + 32 * c;
-        w[c] = idx < hi ? dev::ld_relaxed_u64(P.status + idx) : pad;
-      }
-    }
-    for (int spins = 0;; ++spins) {
-      bool missing = false;
-#pragma unroll
-      for (int c = 0; c < LBW; ++c) missing |= (uint32_t)(w[c] >> 32) != want;
-      if (!__any_sync(0xffffffffu, missing)) break;
-      if (spins > 1) __nanosleep(64);
-#pragma unroll
-      for (int c = 0; c < LBW; ++c)
-        if ((uint32_t)(w[c] >> 32) != want) w[c] = dev::ld_relaxed_u64(P.status + base + lane + 32 * c);
-    }
-    uint32_t v0 = 0, v1 = 0;
-#pragma unroll
-    for (int c = 0; c < LBW; ++c) {
-      v0 += (uint32_t)w[c] & 0xFFFFu;
-      v1 += ((uint32_t)w[c] >> 16) & 0xFFFFu;
-    }
-    t0 += __reduce_add_sync(0xffffffffu, v0);
-    t1 += __reduce_add_sync(0xffffffffu, v1);
-  }
-}
-
 // Compute warps: copy tile k's run of selected rows from the ring to its place
 // (ROWS mode: the run holds row ids).
-template <bool ROWS, int M, typename SM>
+template <bool ROWS, typename SM>
 __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int tid) {
   // tell the look-back warp not to wait for later counts (a monotone hint,
   // relaxed accesses on both sides: never a plain racing access)
@@ -432,21 +346,6 @@ __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int
   const int32_t* run = S.ring + S.start[k % K];  // contiguous, never wraps
   int64_t lim = P.out_cap - g;
   lim = lim < 0 ? 0 : (lim > c ? c : lim);
-  if (M == 2) {  // the second output's run follows the first in the ring
-    const int64_t g2 = S.goff2[k % K];
-    const int32_t c2 = S.cnt2[k % K];
-    int64_t lim2 = P.out_cap2 - g2;
-    lim2 = lim2 < 0 ? 0 : (lim2 > c2 ? c2 : lim2);
-    int32_t* __restrict__ out2 = P.out2 + g2;
-    if (S.spilled[k % K]) {  // from the spill slot (global, L2)
-      // (a batched 16-B readback needs registers the 2-CTA/SM kernel does not
-      // have: it spilled and slowed every pair; measured)
-      const int32_t* sp = P.spill + ((int64_t)blockIdx.x * K + k % K) * SEL_TILE;
-      for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = sp[e];
-    } else {
-      for (int e = tid; e < (int)lim2; e += SEL_THREADS) out2[e] = run[c + e];
-    }
-  }
   if (!ROWS) {
     int32_t* __restrict__ out = P.out + g;
     for (int e = tid; e < (int)lim; e += SEL_THREADS) out[e] = run[e];
@@ -456,11 +355,10 @@ __device__ __forceinline__ void write_tile(SM& S, const SelParams& P, int k, int
   }
 }
 
-template <bool HAS_NE, bool ROWS, int M>
+template <bool HAS_NE, bool ROWS>
 __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams P) {
-  static_assert(M == 1 || (M == 2 && !ROWS), "two outputs in value mode only");
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  using SM = SmemFor<M>;
+  using SM = SelSmem;
   constexpr int RING = SM::kRing;
   SM& S = *reinterpret_cast<SM*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -540,7 +438,6 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ======================= look-back warp: tile offsets =======================
     const uint32_t want = (uint32_t)((FLAG_A | (tag << TAG_SHIFT)) >> 32);
     int64_t my_prefix = 0;  // inclusive prefix of this CTA's last placed tile
-    int64_t my_prefix2 = 0;  // M == 2: the same for the second output
     int64_t t_last = -1;    // tile index of the last window copied
     int m = 0x7fffffff;     // tiles of this CTA, known once the end marker is counted
     // Decisions are warp-uniform: a lane that sees a barrier phase complete has
@@ -587,25 +484,14 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         mbar_wait(&S.winfull[q], (uint32_t)((k / Q) & 1));
         PT_END(6, t0, lane == 0);
         PT_BEGIN(t1);
-        int64_t g, g2 = 0;
-        if constexpr (M == 2) {
-          int64_t w0, w1;
-          window_sum2(S, P, q, lane, want, w0, w1);
-          g = my_prefix + w0;
-          g2 = my_prefix2 + w1;
-          my_prefix2 = g2 + S.cnt2[k % K];
-        } else {
-          g = my_prefix + window_sum(S, P, q, lane, want);
-        }
+        const int64_t g = my_prefix + window_sum(S, P, q, lane, want);
         PT_END(7, t1, lane == 0);
         const int64_t tp = S.whi[q];
         my_prefix = g + S.cnt[k % K];
         if (lane == 0) {
           S.goff[k % K] = g;
-          if (M == 2) S.goff2[k % K] = g2;
           if (tp == ntiles - 1) {  // every tile has published (read the epoch): advance it
             *P.d_count = my_prefix;
-            if (M == 2) *P.d_count2 = my_prefix2;
             st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
           }
           mbar_arrive(&S.placed[k % K]);
@@ -619,10 +505,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       if (atomicAdd(&P.hdr[H_DONE], 1u) == gridDim.x - 1) {
         *P.ticket = 0ull;
         P.hdr[H_DONE] = 0u;
-        if (ntiles == 0) {
-          *P.d_count = 0;
-          if (M == 2) *P.d_count2 = 0;
-        }
+        if (ntiles == 0) *P.d_count = 0;
         // High-water mark of status words this workspace has carried.  When the
         // next launch's 28-bit tag wraps to 0, clear all of them: a word left by
         // a launch exactly 2^28 launches earlier could otherwise read as ready.
@@ -660,16 +543,12 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       for (int j = 0; j < SEL_VEC; ++j) v[j] = base[32 * j + lane];
     }
     const int64_t v0 = t * SEL_TILE + warp * WROWS;
-    uint32_t fl = 0;   // bit 4j+c: row warp*1024 + 4*(32j + lane) + c selected
-    uint32_t fl2 = 0;  // M == 2: the same for the second output
+    uint32_t fl = 0;  // bit 4j+c: row warp*1024 + 4*(32j + lane) + c selected
     if (v0 >= P.mis && v0 + WROWS <= nv) {
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          fl |= (uint32_t)keep<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
-          if (M == 2) fl2 |= (uint32_t)keep2<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
-        }
+        for (int c = 0; c < 4; ++c) fl |= (uint32_t)keep<HAS_NE>(comp(v[j], c), P) << (4 * j + c);
     } else {
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
@@ -678,7 +557,6 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         for (int c = 0; c < 4; ++c) {
           const bool in = (e0 + c >= P.mis) & (e0 + c < nv);
           fl |= (uint32_t)(keep<HAS_NE>(comp(v[j], c), P) & in) << (4 * j + c);
-          if (M == 2) fl2 |= (uint32_t)(keep2<HAS_NE>(comp(v[j], c), P) & in) << (4 * j + c);
         }
       }
     }
@@ -686,71 +564,48 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ---- buffer: order (warp, j, lane, c); packed per-j counts, warp scans.
     // SWAR popcount of each nibble of fl (nibble j = the lane's 4 rows of
     // vector j), then j goes to word j&1, byte j>>1 (8 bits: a warp total <= 128).
-    // M == 2: words NPK.. hold the second output's counts.
-    constexpr int NQ = NPK * M;
-    uint32_t packed[NQ], inc[NQ], tot[NQ];
-#pragma unroll
-    for (int o = 0; o < M; ++o) {
-      const uint32_t f = o == 0 ? fl : fl2;
-      uint32_t x = f - ((f >> 1) & 0x55555555u);
+    uint32_t packed[NPK], inc[NPK], tot[NPK];
+    {
+      uint32_t x = fl - ((fl >> 1) & 0x55555555u);
       x = (x & 0x33333333u) + ((x >> 2) & 0x33333333u);
       if (NPK == 2) {  // even j in word 0, odd j in word 1, byte j >> 1
-        packed[NPK * o] = x & 0x0F0F0F0Fu;
-        packed[NPK * o + 1] = (x >> 4) & 0x0F0F0F0Fu;
+        packed[0] = x & 0x0F0F0F0Fu;
+        packed[NPK - 1] = (x >> 4) & 0x0F0F0F0Fu;
       } else {  // 16 flag bits: bytes j0, j2, j1, j3
-        packed[NPK * o] = (x & 0x0F0Fu) | (((x >> 4) & 0x0F0Fu) << 16);
+        packed[0] = (x & 0x0F0Fu) | (((x >> 4) & 0x0F0Fu) << 16);
       }
 #pragma unroll
-      for (int q = 0; q < NPK; ++q) inc[NPK * o + q] = packed[NPK * o + q];
+      for (int q = 0; q < NPK; ++q) inc[q] = packed[q];
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
 #pragma unroll
-      for (int q = 0; q < NQ; ++q) {
+      for (int q = 0; q < NPK; ++q) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, inc[q], d);
         if (lane >= d) inc[q] += y;
       }
     }
-    uint32_t wtotal[M];
+    uint32_t wtotal = 0;
 #pragma unroll
-    for (int o = 0; o < M; ++o) wtotal[o] = 0;
-#pragma unroll
-    for (int q = 0; q < NQ; ++q) {
+    for (int q = 0; q < NPK; ++q) {
       tot[q] = __shfl_sync(0xffffffffu, inc[q], 31);  // per-row warp totals (<= 128 each)
-      wtotal[q / NPK] += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
+      wtotal += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
     }
-    if (lane == 0) {
-#pragma unroll
-      for (int o = 0; o < M; ++o) S.wtot[i & 1][o][warp] = wtotal[o];
-    }
+    if (lane == 0) S.wtot[i & 1][warp] = wtotal;
     PT_BEGIN(tb);
     compute_bar();  // B1: wtot visible; every warp is done with this tile's input slot
     PT_END(3, tb, tid == 0);
     PT_END(13, tb, tid == 224);
-    const uint32_t wt = lane < NW ? S.wtot[i & 1][0][lane] : 0u;
+    const uint32_t wt = lane < NW ? S.wtot[i & 1][lane] : 0u;
     const int32_t agg = (int32_t)__reduce_add_sync(0xffffffffu, wt);
     const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
-    int32_t agg2 = 0, wbase2 = 0;
-    if (M == 2) {
-      const uint32_t wt2 = lane < NW ? S.wtot[i & 1][1][lane] : 0u;
-      agg2 = (int32_t)__reduce_add_sync(0xffffffffu, wt2);
-      wbase2 = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt2 : 0u);
-    }
-    // M == 2: when both runs together exceed the ring (both outputs keep most
-    // of the tile), the second run goes to this CTA's global spill slot for
-    // the tile (read back when the tile is written).  Measured: spilling both
-    // runs, or placing such tiles straight from registers after waiting for
-    // their own placement, is slower still.
-    const bool spill2 = M == 2 && agg + agg2 > RA_SEL_SPILL_AT;
     if (ROWS && P.meta && lane == 0) P.meta[t * 12 + warp] = (uint32_t)wbase;
     const bool ring_rows = !ROWS || P.rowids;  // ROWS without ids: placement only, no ring
-    const int32_t rows_in = ring_rows ? agg + (spill2 ? 0 : agg2) : 0;  // ring rows this tile needs
+    const int32_t rows_in = ring_rows ? agg : 0;  // ring rows this tile needs
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
       mbar_arrive(&S.empty[slot]);  // input slot free: the producer refills it
-      const uint64_t aggw = M == 2 ? ((uint64_t)agg | ((uint64_t)agg2 << 16)) : (uint64_t)agg;
-      dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | aggw);
+      dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
       S.cnt[i % K] = agg;
-      if (M == 2) S.cnt2[i % K] = agg2;
       S.tidx[i % K] = t;
       mbar_arrive(&S.counted[i % K]);
     }
@@ -774,41 +629,23 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         start = wp;
         break;
       }
-      write_tile<ROWS, M, SM>(S, P, head, tid);
-      used -= ring_rows ? S.cnt[head % K] + (M == 2 && !S.spilled[head % K] ? S.cnt2[head % K] : 0) : 0;
+      write_tile<ROWS, SM>(S, P, head, tid);
+      used -= ring_rows ? S.cnt[head % K] : 0;
       ++head;
       forced = true;
     }
     if (forced) compute_bar();  // rows written out are read before they are overwritten
-    if (tid == 0) {
-      S.start[i % K] = start;
-      if (M == 2) S.spilled[i % K] = spill2;
-    }
+    if (tid == 0) S.start[i % K] = start;
     used += rows_in;
-    // ---- scatter the tile into the ring (M == 2: the second run after the first)
-#pragma unroll
-    for (int o = 0; o < (ring_rows ? M : 0); ++o) {
-      const uint32_t f = o == 0 ? fl : fl2;
-      int32_t rb = start + (o == 0 ? wbase : agg + wbase2);
+    // ---- scatter the tile into the ring
+    if (ring_rows) {
+      int32_t rb = start + wbase;
 #if RA_SEL_PTXSCATTER
       const uint32_t ring0 = smem_u32(S.ring);
 #endif
-      if (M == 2 && o == 1 && spill2) {  // second run -> the tile's spill slot (global)
-        int32_t* slot = P.spill + ((int64_t)blockIdx.x * K + i % K) * SEL_TILE;
-        rb = wbase2;
-#pragma unroll
-        for (int j = 0; j < SEL_VEC; ++j) {
-          const int q = NPK * o + q_of(j);
-          int32_t* a = slot + rb + (int32_t)(((inc[q] - packed[q]) >> (8 * b_of(j))) & 0xFFu);
-#pragma unroll
-          for (int c = 0; c < 4; ++c) put_if_global(a, f, 1u << (4 * j + c), comp(v[j], c));
-          rb += (int32_t)((tot[q] >> (8 * b_of(j))) & 0xFFu);
-        }
-        continue;
-      }
 #pragma unroll
       for (int j = 0; j < SEL_VEC; ++j) {
-        const int q = NPK * o + q_of(j);
+        const int q = q_of(j);
         const uint32_t ex = inc[q] - packed[q];
         int32_t p = rb + (int32_t)((ex >> (8 * b_of(j))) & 0xFFu);
 #if RA_SEL_PTXSCATTER
@@ -818,10 +655,10 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
           // ROWS: the row id (n < 2^32 is checked by ra_select_rows)
           const int32_t val = ROWS ? (int32_t)(uint32_t)(t * SEL_TILE + warp * WROWS - P.mis + 4 * (32 * j + lane) + c)
                                    : comp(v[j], c);
-          put_if(a, f, 1u << (4 * j + c), val);
+          put_if(a, fl, 1u << (4 * j + c), val);
         }
 #else
-        const uint32_t bits = (f >> (4 * j)) & 0xFu;
+        const uint32_t bits = (fl >> (4 * j)) & 0xFu;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
           if (bits & (1u << c))
@@ -834,8 +671,8 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     wp = start + rows_in;
     // ---- gather: tile i - LAG is due
     if (i - LAG >= head) {
-      write_tile<ROWS, M, SM>(S, P, head, tid);
-      used -= ring_rows ? S.cnt[head % K] + (M == 2 && !S.spilled[head % K] ? S.cnt2[head % K] : 0) : 0;
+      write_tile<ROWS, SM>(S, P, head, tid);
+      used -= ring_rows ? S.cnt[head % K] : 0;
       ++head;
     }
   }
@@ -846,20 +683,20 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     mbar_arrive(&S.counted[i % K]);
   }
   compute_bar();  // scatters of the last tiles are visible
-  for (; head < i; ++head) write_tile<ROWS, M, SM>(S, P, head, tid);
+  for (; head < i; ++head) write_tile<ROWS, SM>(S, P, head, tid);
 }
 
 // smem opt-in + occupancy of each instantiation, once per device
-template <bool HAS_NE, bool ROWS, int M>
+template <bool HAS_NE, bool ROWS>
 int ensure_config(int dev, int& per_sm) {
   static std::atomic<int> cfg[64];
   const int v = device_once(cfg, dev, [] {
-    const int smem = (int)sizeof(SmemFor<M>);
-    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE, ROWS, M>,
+    const int smem = (int)sizeof(SelSmem);
+    cudaError_t e = cudaFuncSetAttribute(select_fused_kernel<HAS_NE, ROWS>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(select smem)");
     int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE, ROWS, M>, BLOCK, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, select_fused_kernel<HAS_NE, ROWS>, BLOCK, smem);
     if (e != cudaSuccess) return cuda_fail(e, "occupancy(select)");
     if (occ < 1) return fail(RA_E_CUDA, "select kernel does not fit on an SM");
     return occ;
@@ -875,12 +712,6 @@ int64_t sel_max_tiles(int64_t n) { return (n + 3 + SEL_TILE - 1) / SEL_TILE + 1;
 
 size_t sel_status_bytes(int64_t n) { return SEL_HDR_BYTES + 8 * (size_t)sel_max_tiles(n) + 16; }
 
-size_t sel_spill_bytes(int64_t n) {
-  int64_t g = sel_max_tiles(n);
-  if (g > SEL_MULTI_MAX_GRID) g = SEL_MULTI_MAX_GRID;
-  return (size_t)g * K * SEL_TILE * 4;
-}
-
 size_t sel_inter_bytes(int64_t n) {
   // two int32[n] relations + two int64 counts, 256-B granules
   const size_t rel = (((size_t)(n > 0 ? n : 1) * 4 + 255) / 256) * 256;
@@ -890,42 +721,17 @@ size_t sel_inter_bytes(int64_t n) {
 int sel_ctas_per_sm() {
   const int dev = current_device();
   int per_sm = 0;
-  if (ensure_config<false, false, 1>(dev, per_sm)) return -1;
+  if (ensure_config<false, false>(dev, per_sm)) return -1;
   return per_sm;
 }
 
 int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, const CanonPred& cp,
                        int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
-                       cudaStream_t s, uint32_t* rows, const SelSecond* second, const SelMasks* masks) {
+                       cudaStream_t s, uint32_t* rows, const SelMasks* masks) {
   SelParams P;
   P.rowids = rows;
   P.fmask = masks ? masks->fmask : nullptr;
   P.meta = masks ? masks->meta : nullptr;
-  P.lo2 = 0;
-  P.span2 = 0;
-  P.n_ne2 = 0;
-  for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne2[j] = 0;
-  P.out2 = nullptr;
-  P.spill = nullptr;
-  P.out_cap2 = 0;
-  P.d_count2 = nullptr;
-  if (second) {
-    const CanonPred& c2 = second->cp;
-    P.lo2 = c2.lo;
-    P.span2 = (uint32_t)c2.hi - (uint32_t)c2.lo;
-    P.n_ne2 = c2.n_ne;
-    for (int j = 0; j < RA_MAX_PREDS; ++j) P.ne2[j] = j < c2.n_ne ? c2.ne[j] : 0;
-    if (c2.lo > c2.hi) {  // empty interval
-      P.lo2 = 0;
-      P.span2 = 0;
-      P.n_ne2 = 1;
-      P.ne2[0] = 0;
-    }
-    P.out2 = second->out;
-    P.spill = second->spill;
-    P.out_cap2 = second->out_cap;
-    P.d_count2 = second->d_count;
-  }
   const uintptr_t a = (uintptr_t)d_in;
   P.mis = (int32_t)((a & 15u) >> 2);
   P.abase = (const int32_t*)(a - (a & 15u));
@@ -949,27 +755,21 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
   }
   if (n_max >= ((int64_t)1 << 34)) return fail(RA_E_INVAL, "n=%lld >= 2^34", (long long)n_max);
   const int dev = current_device();
-  const bool ne = P.n_ne > 0 || P.n_ne2 > 0;
+  const bool ne = P.n_ne > 0;
   const bool rw = rows != nullptr || masks != nullptr;
-  const bool two = second != nullptr;
-  if (rw && two) return fail(RA_E_INVAL, "row-id mode has one output");
   int per_sm = 1;
   int rc;
   const void* kern;
-  if (two) {
-    rc = ne ? ensure_config<true, false, 2>(dev, per_sm) : ensure_config<false, false, 2>(dev, per_sm);
-    kern = ne ? (const void*)select_fused_kernel<true, false, 2> : (const void*)select_fused_kernel<false, false, 2>;
-  } else if (rw) {
-    rc = ne ? ensure_config<true, true, 1>(dev, per_sm) : ensure_config<false, true, 1>(dev, per_sm);
-    kern = ne ? (const void*)select_fused_kernel<true, true, 1> : (const void*)select_fused_kernel<false, true, 1>;
+  if (rw) {
+    rc = ne ? ensure_config<true, true>(dev, per_sm) : ensure_config<false, true>(dev, per_sm);
+    kern = ne ? (const void*)select_fused_kernel<true, true> : (const void*)select_fused_kernel<false, true>;
   } else {
-    rc = ne ? ensure_config<true, false, 1>(dev, per_sm) : ensure_config<false, false, 1>(dev, per_sm);
-    kern = ne ? (const void*)select_fused_kernel<true, false, 1> : (const void*)select_fused_kernel<false, false, 1>;
+    rc = ne ? ensure_config<true, false>(dev, per_sm) : ensure_config<false, false>(dev, per_sm);
+    kern = ne ? (const void*)select_fused_kernel<true, false> : (const void*)select_fused_kernel<false, false>;
   }
   if (rc) return rc;
   const int64_t ntiles_max = n_max > 0 ? (n_max + P.mis + SEL_TILE - 1) / SEL_TILE : 0;
   int64_t grid = (int64_t)num_sms() * per_sm;
-  if (two && grid > SEL_MULTI_MAX_GRID) grid = SEL_MULTI_MAX_GRID;  // spill slots exist for this many CTAs
   // RA_SEL_MAX_CTAS (diagnostics only): cap the grid, for the paper's Fig 12
   // experiment (a SELECT with half the CTAs, two of them on two streams)
   static const int64_t max_ctas = getenv("RA_SEL_MAX_CTAS") ? atoll(getenv("RA_SEL_MAX_CTAS")) : 0;

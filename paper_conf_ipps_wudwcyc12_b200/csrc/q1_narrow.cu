@@ -51,6 +51,9 @@ namespace ra {
 #ifndef RA_Q1N_PRMT
 #define RA_Q1N_PRMT 1
 #endif
+#ifndef RA_Q1N_WSLICE
+#define RA_Q1N_WSLICE 1  // per-warp 64-bit flush sums (plain adds) instead of CTA-wide shared atomics
+#endif
 
 namespace {
 
@@ -97,7 +100,11 @@ struct QnSmem {
 #else
   uint4 rec[NS + 1][2][QN_NT];  // [slot][half][thread]: thread-private 32-byte records
 #endif
+#if RA_Q1N_WSLICE
+  unsigned long long wsum[QN_NW][NS][6];  // per-warp sums: count, qty, price, disc, disc_price, charge
+#else
   unsigned long long wsum[NS][6];  // CTA sums: count, qty, price, disc, disc_price, charge
+#endif
   uint64_t full[QN_STAGES], empty[QN_STAGES];
   uint32_t status;
   bool last;
@@ -249,12 +256,22 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
     const unsigned long long dph = warp_sum32(a.w), dpl = warp_sum32(b.x);
     const unsigned long long chh = warp_sum32(b.y), chl = warp_sum32(b.z);
     if (lane == 0) {
+#if RA_Q1N_WSLICE  // this warp's own sums: plain 64-bit adds (64-bit shared atomics are CAS loops)
+      unsigned long long* w = S.wsum[threadIdx.x >> 5][s];
+      w[0] += cnt;
+      w[1] += q;
+      w[2] += p;
+      w[3] += disc;
+      w[4] += (dph << 16) + dpl;
+      w[5] += 100ull * ((dph << 16) + dpl) + (chh << 16) + chl;  // 100 dp + tax dp
+#else
       atomicAdd(&S.wsum[s][0], cnt);
       atomicAdd(&S.wsum[s][1], q);
       atomicAdd(&S.wsum[s][2], p);
       atomicAdd(&S.wsum[s][3], disc);
       atomicAdd(&S.wsum[s][4], (dph << 16) + dpl);
       atomicAdd(&S.wsum[s][5], 100ull * ((dph << 16) + dpl) + (chh << 16) + chl);  // 100 dp + tax dp
+#endif
     }
 #if RA_Q1N_RED
 #pragma unroll
@@ -290,7 +307,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
 #endif
     }
   }
-  if (tid < NS * 6) (&S.wsum[0][0])[tid] = 0ull;
+  for (int i = tid; i < (int)(sizeof(S.wsum) / 8); i += blockDim.x) reinterpret_cast<unsigned long long*>(S.wsum)[i] = 0ull;
   if (tid == 0) S.status = 0;
   __syncthreads();
 
@@ -363,22 +380,18 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
   }
   // CTA partial -> P.blocks[blockIdx]; the last CTA folds all of them
   __syncthreads();
-  if (tid < NS * 4) {
-    const int sl = tid >> 2, f = tid & 3;
+  if (tid < NS * 6) {  // CTA sums (of the warps' sums) -> P.blocks[blockIdx]: v = {cnt, qty, price, disc, dp lo/hi, ch lo/hi}
+    const int sl = tid / 6, f = tid % 6;
+#if RA_Q1N_WSLICE
+    unsigned long long v = 0;
+    for (int w = 0; w < QN_NW; ++w) v += S.wsum[w][sl][f];
+#else
+    const unsigned long long v = S.wsum[sl][f];
+#endif
     Q1Block* mine = P.blocks + blockIdx.x;
-    if (f == 0) {
-      mine->v[sl][0] = S.wsum[sl][0];
-      mine->v[sl][1] = S.wsum[sl][1];
-    } else if (f == 1) {
-      mine->v[sl][2] = S.wsum[sl][2];
-      mine->v[sl][3] = S.wsum[sl][3];
-    } else if (f == 2) {
-      mine->v[sl][4] = S.wsum[sl][4];
-      mine->v[sl][5] = 0;
-    } else {
-      mine->v[sl][6] = S.wsum[sl][5];
-      mine->v[sl][7] = 0;
-    }
+    static constexpr int DST[6] = {0, 1, 2, 3, 4, 6};
+    mine->v[sl][DST[f]] = v;
+    if (f >= 4) mine->v[sl][DST[f] + 1] = 0;
   }
   if (tid == 0) P.blocks[blockIdx.x].status = S.status;
   publish_and_fold(P, &S.last);

@@ -1,8 +1,5 @@
-# narrow Q1 variants: rebuild libra.so with extra defines, time SF10/SF100 (scripts/prof_driver.py q1time)
+# narrow Q1: per-warp flush sums vs CTA shared 64-bit atomics; parity + timings
 mkdir -p gpurun_out
-NVF0="-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-fvisibility=hidden -shared -Xptxas -v --expt-relaxed-constexpr"
-for defs in "$@"; do
-  make -s -B paper_conf_ipps_wudwcyc12_b200/libra.so "NVFLAGS=$NVF0 $defs" >/dev/null 2>&1 || { echo "build $defs FAILED"; continue; }
-  echo "== $defs"; python scripts/prof_driver.py q1time 20 2>&1 | grep narrow
-done
-make -s -B all >/dev/null 2>&1
+timeout -s KILL 600 python -m pytest tests/test_q1_narrow_gpu.py tests/test_q1_gpu.py -x -q -p no:cacheprovider 2>&1 | tail -2
+( timeout -s KILL 300 python scripts/prof_driver.py q1time 20
+  RA_LIB_PATH=$PWD/build/libra_q1nold.so timeout -s KILL 300 python scripts/prof_driver.py q1time 20 ) 2>&1 | tee gpurun_out/q1n_ab.txt

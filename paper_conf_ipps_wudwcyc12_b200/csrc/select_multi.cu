@@ -64,6 +64,12 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 #define RA_MO_REGS 88
 #define RA_MO_AUXREGS 56
 #endif
+#ifndef RA_MO_SCAT_ARRIVALS
+// arrivals per tile on `scattered`: every compute thread releases its own ring
+// writes (the form compute-sanitizer's racecheck models; one warp-wide arrive
+// per warp, measured the same speed as lane 0 after __syncwarp, =GW)
+#define RA_MO_SCAT_ARRIVALS GT
+#endif
 #ifndef RA_MO_TMA
 #define RA_MO_TMA 0  // writer: TMA bulk tensor stores instead of warp stores
 #endif
@@ -427,7 +433,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
     for (int s = 0; s < K; ++s) {
       mbar_init(&S.counted[s], 1);
       mbar_init(&S.placed[s], 1);
-      mbar_init(&S.scattered[s], GW);
+      mbar_init(&S.scattered[s], RA_MO_SCAT_ARRIVALS);
       mbar_init(&S.written[s], 1);
       mbar_init(&S.allocd[s], 1);
     }
@@ -649,7 +655,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
       PROF_ADD(16, t_wr);
       if (wt == 0) {
         PROF_LAT(19, S.t_placed[k % K]);
-        st_relaxed_shared(&S.w_done, k + 1);
+        st_release_shared(&S.w_done, k + 1);  // the ring reads above happen-before a reuse of the space
         mbar_arrive(&S.written[k % K]);  // release: the ring space
       }
     }
@@ -754,7 +760,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
       const int64_t vend = s0 + rows_in;
       while (true) {
         // h = tiles written so far (>= i - K + 1: tile i - K is written)
-        const int32_t h = ld_relaxed_shared(&S.w_done);
+        const int32_t h = ld_acquire_shared(&S.w_done);
         if (h >= i || vend - S.vstart[h % K] <= RING) break;
         st_relaxed_shared(&S.demand, h);  // the look-back places tile h without delay
         MWAIT(&S.written[h % K], (uint32_t)((h / K) & 1), 10, (int)h);
@@ -809,7 +815,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
       rb += (agg[o] + 31) & ~31;
     }
     __syncwarp();
-    if (lane == 0) mbar_arrive(&S.scattered[i % K]);
+    if (RA_MO_SCAT_ARRIVALS == GT || lane == 0) mbar_arrive(&S.scattered[i % K]);
     PROF_ADD(15, t_sc);
     PROF_ADD(11, t_it);
   }

@@ -569,7 +569,10 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                               "rows": 1 << 30, "rows_per_s": (1 << 30) / (bms * 1e-3), "ms_per_step": bms,
                               "kernel_ms": bkms, "scaling": "strong",
                               "roofline": {"kernel": "select_multi_kernel<M=1>", "bound": "hbm", "achieved": bach,
-                                           "peak": peak, "unit": "GB/s", "frac": bach / peak}}
+                                           "peak": peak, "unit": "GB/s", "frac": bach / peak,
+                                           "algorithmic_bytes_per_launch": 4 * nb + 4 * bk,
+                                           "traffic": ncu_traffic(f"select_chain_k{k}_s{s_sel}_n{nb.bit_length() - 1}")
+                                           if nb & (nb - 1) == 0 else None}}
     del xb, ob, wsb
 
     # --- f2: several SELECTs filtering the same input (Fig 2(c)): one fused pass

@@ -107,6 +107,9 @@ constexpr int BLOCK = SEL_THREADS + 64;  // + the look-back and producer warps
 #endif
 constexpr int LAG = RA_SEL_LAG;          // tile k is written when tile k+LAG is counted (or earlier)
 constexpr int K = LAG + 2;               // metadata slots: tiles counted but not yet written
+#ifndef RA_SEL_SMALL_ROWS_DEFAULT
+#define RA_SEL_SMALL_ROWS_DEFAULT (1ll << 21)  // fused chains up to this many rows run select_fused_kernel
+#endif
 #ifndef RA_SEL_PDL
 #define RA_SEL_PDL 1
 #endif
@@ -803,10 +806,17 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
                       size_t ws_bytes, cudaStream_t s) {
   if (fused || k <= 1) {
     // the fused chain is one output of the warp-specialised multi-output pass
-    // (select_multi.cu): one kernel, writer warps, cooperative look-back
+    // (select_multi.cu): one kernel, writer warps, cooperative look-back.
+    // Small inputs (a few tiles per SM) are launch/latency-bound: the lighter
+    // single-output kernel of this file starts faster there (both produce the
+    // same result; same workspace layout for one output).  RA_SEL_SMALL_ROWS
+    // (diagnostics) moves the threshold.
+    static const int64_t small_rows =
+        getenv("RA_SEL_SMALL_ROWS") ? atoll(getenv("RA_SEL_SMALL_ROWS")) : RA_SEL_SMALL_ROWS_DEFAULT;
     CanonPred cp;
     int rc = canonicalize(h_preds, k, &cp);
     if (rc) return rc;
+    if (n <= small_rows) return launch_select_pass(d_in, n, nullptr, cp, d_out, out_cap, d_count, d_ws, s, nullptr);
     return launch_select_multi(d_in, n, &cp, 1, &d_out, &out_cap, &d_count, d_ws, s);
   }
   // Unfused composition: one pass per predicate, intermediates at the end of

@@ -70,6 +70,9 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 // per warp, measured the same speed as lane 0 after __syncwarp, =GW)
 #define RA_MO_SCAT_ARRIVALS GT
 #endif
+#ifndef RA_MO_SPLIT
+#define RA_MO_SPLIT 0  // 1: publish (gtid 0) and ring allocation (gtid 32) by two warps
+#endif
 #ifndef RA_MO_TMA
 #define RA_MO_TMA 0  // writer: TMA bulk tensor stores instead of warp stores
 #endif
@@ -739,15 +742,19 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
         const uint64_t a = (uint64_t)(uint32_t)agg[2 * j] | ((2 * j + 1 < M ? (uint64_t)(uint32_t)agg[2 * j + 1] : 0ull) << 16);
         dev::st_relaxed_u64(P.status + t * W + j, FLAG_A | (tag << TAG_SHIFT) | a);
       }
-      int32_t rows_in = 0;  // the tile's runs, each padded to a multiple of 32 rows (128-B aligned starts)
+      // (the tile's runs are each padded to a multiple of 32 rows: 128-B aligned starts)
 #pragma unroll
-      for (int o = 0; o < M; ++o) {
-        S.cnt[i % K][o] = agg[o];
-        rows_in += (agg[o] + 31) & ~31;
-      }
+      for (int o = 0; o < M; ++o) S.cnt[i % K][o] = agg[o];
       S.tidx[i % K] = t;
       PROF_STAMP(S.t_count[i % K]);
       mbar_arrive(&S.counted[i % K]);
+      PROF_ADD(13, t_g0);
+    }
+    if (gtid == (RA_MO_SPLIT ? 32 : 0)) {  // (RA_MO_SPLIT: another warp allocates while gtid 0 publishes)
+      int32_t rows_in = 0;
+#pragma unroll
+      for (int o = 0; o < M; ++o) rows_in += (agg[o] + 31) & ~31;
+      if (RA_MO_SPLIT && i >= K) MWAIT(&S.written[i % K], (uint32_t)(((i / K) - 1) & 1), 8, (int)i);
       // ---- allocate the tile's runs, in CTA tile order (after tile i-1's).
       // Virtual ring coordinates grow monotonically; a run set that would
       // cross the physical end starts at the next multiple of RING.  Pending
@@ -769,7 +776,6 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
       S.vstart[i % K] = s0;
       S.a_va = vend;
       mbar_arrive(&S.allocd[i % K]);
-      PROF_ADD(13, t_g0);
     }
     PROF_T0(t_b2);
     group_bar(g);  // B2: the run start is visible

@@ -20,6 +20,8 @@ os.makedirs(OUT, exist_ok=True)
 CAPTURES = {  # report -> (summary name, traffic key, command)
     "prof_select": ("select_chain_k2_s05_n28", "select_chain_k2_s0.5_n28",
                     "python scripts/prof_driver.py select 5  (2^28 int32, k=2, s=0.5/stage; select_multi_kernel<1>)"),
+    "prof_select_n30": ("select_chain_k2_s05_n30", "select_chain_k2_s0.5_n30",
+                        "python scripts/prof_driver.py select 3 30  (2^30 int32, k=2, s=0.5/stage; select_multi_kernel<1>)"),
     "prof_select_s01": ("select_chain_k1_s001_n28", "select_chain_k1_s0.01_n28",
                         "python scripts/prof_driver.py select 5 28 1 0.01  (2^28 int32, k=1, s=0.01; select_multi_kernel<1>)"),
     "prof_select_s09": ("select_chain_k1_s09_n28", "select_chain_k1_s0.9_n28",

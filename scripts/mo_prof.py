@@ -23,7 +23,9 @@ x = torch.empty(n, dtype=torch.int32, device="cuda")
 ragen.int32_column_dev(2, x)
 outs = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
 buf = (ctypes.c_ulonglong * 64)()
-for M, s in [(1, 0.01), (1, 0.5), (2, 0.5), (2, 0.9), (3, 0.01)]:
+CASES = {"m1": [(1, 0.01), (1, 0.25)], "dense": [(2, 0.9), (4, 0.9), (4, 0.5)]}.get(
+    os.environ.get("MO_PROF_CASES", ""), [(1, 0.01), (1, 0.5), (2, 0.5), (2, 0.9), (3, 0.01)])
+for M, s in CASES:
     ch = [[("lt", ragen.nested_thresholds(s, 1)[0])]] * M
     for _ in range(3):
         R.select_multi(x, ch, outs=outs[:M])

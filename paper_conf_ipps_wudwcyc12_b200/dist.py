@@ -88,3 +88,36 @@ def gather_partials(partial, group=None):
     world = dist.get_world_size(group)
     out = torch.empty(world * partial.numel(), dtype=torch.uint8, device=partial.device)
     return _all_gather(out, partial, group)
+
+
+def gather_outputs(out, count, offsets, total, root: int = 0, group=None):
+    """Optional concatenation of the sharded SELECT output onto one rank
+    (SURVEY §8(e)): rank r sends its rows out[:count_r] to `root`, which
+    receives them at their global offsets (from ``exchange_counts``) into one
+    tensor of ``total`` rows, in rank order — equal to the 1-GPU result.
+    Point-to-point transfers (NCCL send/recv over NVLink on the GPU box, gloo
+    in tests).  Returns the concatenation on `root`, None elsewhere."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    c = int(count)
+    staged = out.is_cuda and dist.get_backend(group) == "gloo"  # gloo: point-to-point on host tensors
+    if rank != root:
+        if c:
+            dist.send(out[:c].cpu() if staged else out[:c].contiguous(), dst=root, group=group)
+        return None
+    offs = [int(v) for v in (offsets.tolist() if hasattr(offsets, "tolist") else offsets)]
+    tot = int(total)
+    bounds = offs[1:] + [tot]
+    full = torch.empty(max(1, tot), dtype=out.dtype, device=out.device)[:tot]
+    full[offs[root]:offs[root] + c].copy_(out[:c])
+    for r in range(world):
+        if r != root and bounds[r] > offs[r]:
+            if staged:
+                tmp = torch.empty(bounds[r] - offs[r], dtype=out.dtype)
+                dist.recv(tmp, src=r, group=group)
+                full[offs[r]:bounds[r]].copy_(tmp)
+            else:
+                dist.recv(full[offs[r]:bounds[r]], src=r, group=group)
+    return full

@@ -70,6 +70,10 @@ def _worker(rank, world, port, q):
         dist.all_reduce(buf)  # assemble for checking only
         whole = oracle.select(x, preds)
         ok_select = bool(np.array_equal(buf.numpy(), whole))
+        # optional concatenation onto rank 0 (point-to-point), in rank order
+        offs = rdist.exclusive_offsets(counts.tolist())
+        full = rdist.gather_outputs(torch.from_numpy(np.ascontiguousarray(mine)), mine.size, offs, total)
+        ok_select &= (full is None) if rank != 0 else bool(np.array_equal(full.numpy(), whole))
         # Q1: shard partials -> all_gather -> exact merge in ra_q1_finalize
         m = 200_001
         cols = ragen.lineitem(22, m, 20000)

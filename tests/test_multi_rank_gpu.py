@@ -55,6 +55,9 @@ def _worker(rank, world, port, n, m, q):
         ok_select = placed.numel() == whole.size and bool(np.array_equal(placed.numpy(), whole))
         host_offs = rdist.exclusive_offsets(counts.tolist())
         ok_offsets = o == host_offs[rank] and t == sum(counts.tolist())
+        offs_dev = torch.tensor(host_offs, dtype=torch.int64, device="cuda")
+        full = rdist.gather_outputs(out, c, offs_dev, t)  # concatenation onto rank 0
+        ok_select &= (full is None) if rank != 0 else bool(np.array_equal(full.cpu().numpy(), whole))
         # ---- Q1 on this rank's rows of one lineitem table
         a, b = rdist.shard_range(m, rank, world)
         cols = ragen.lineitem(62, m, 20000)

@@ -222,27 +222,32 @@ def test_full_size_bench_config(R):
 
 
 
-def test_two_outputs_past_2_pow_31_rows_closed_form(R):
-    """n = 2^31 + 2^28 rows with key[i] = int32(i) (wrapping): output 0 keeps
+@pytest.mark.parametrize("M", [2, 4])
+def test_outputs_past_2_pow_31_rows_closed_form(R, M):
+    """n = 2^31 + 2^28 rows with key[i] = int32(i) (wrapping).  Outputs:
     key >= 0 (rows 0 .. 2^31-1: 2^31 outputs, the last at position 2^31 - 1),
-    output 1 keeps key < 2^30 (rows 0 .. 2^30-1, then the wrapped rows 2^31 ..
-    n-1); both outputs keep whole tiles for 2^30 rows.  Counts exact,
-    sampled outputs against the closed form."""
+    key < 2^30 (rows 0 .. 2^30-1, then the wrapped rows 2^31 .. n-1),
+    key < 0 (the wrapped rows), key >= 2^30 (rows 2^30 .. 2^31-1).  Counts
+    exact (64-bit offsets past 2^31), sampled outputs against the closed form."""
     n = (1 << 31) + (1 << 28)
     x = torch.empty(n, dtype=torch.int32, device="cuda")
     step = 1 << 28
     for lo in range(0, n, step):
         x[lo:lo + step].copy_(torch.arange(lo, lo + step, dtype=torch.int64, device="cuda").to(torch.int32))
-    outs, cnt = R.select_multi(x, [[("ge", 0)], [("lt", 1 << 30)]])
+    chains = [[("ge", 0)], [("lt", 1 << 30)], [("lt", 0)], [("ge", 1 << 30)]][:M]
+    outs, cnt = R.select_multi(x, chains)
     torch.cuda.synchronize()
-    c0, c1 = (int(v) for v in cnt.cpu().tolist())
-    assert (c0, c1) == (1 << 31, (1 << 30) + (1 << 28))
+    del x
+    cs = [int(v) for v in cnt.cpu().tolist()][:M]
+    exp_counts = [1 << 31, (1 << 30) + (1 << 28), 1 << 28, 1 << 30][:M]
+    assert cs == exp_counts
+    closed = [lambda p: p,
+              lambda p: np.where(p < (1 << 30), p, p - (1 << 30) + (1 << 31) - (1 << 32)),
+              lambda p: p - (1 << 31),
+              lambda p: p + (1 << 30)]
     rng = np.random.default_rng(2)
-    for o, c in ((0, c0), (1, c1)):
+    for o in range(M):
+        c = cs[o]
         pos = np.concatenate([np.arange(64), rng.integers(0, c, 1 << 16), np.arange(c - 64, c)])
         got = outs[o][torch.from_numpy(pos).cuda()].cpu().numpy().astype(np.int64)
-        if o == 0:
-            exp = pos
-        else:
-            exp = np.where(pos < (1 << 30), pos, pos - (1 << 30) + (1 << 31) - (1 << 32))
-        np.testing.assert_array_equal(got, exp)
+        np.testing.assert_array_equal(got, closed[o](pos))

@@ -33,8 +33,6 @@
 // its high half carries this launch's tag, so no per-call memset (select_fused
 // uses the same scheme; see there for the look-back's lag and windows).
 
-#include <cuda.h>
-#include <cudaTypedefs.h>
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
@@ -69,12 +67,6 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 // writes (the form compute-sanitizer's racecheck models; one warp-wide arrive
 // per warp, measured the same speed as lane 0 after __syncwarp, =GW)
 #define RA_MO_SCAT_ARRIVALS GT
-#endif
-#ifndef RA_MO_SPLIT
-#define RA_MO_SPLIT 0  // 1: publish (gtid 0) and ring allocation (gtid 32) by two warps
-#endif
-#ifndef RA_MO_TMA
-#define RA_MO_TMA 0  // writer: TMA bulk tensor stores instead of warp stores
 #endif
 #ifndef RA_MO_WU
 #define RA_MO_WU 8  // writer: ring loads in flight per lane
@@ -128,14 +120,6 @@ __host__ __device__ constexpr int q_of(int npk, int j) { return npk == 2 ? (j & 
 __host__ __device__ constexpr int b_of(int npk, int j) { return npk == 2 ? (j >> 1) : ((j >> 1) | ((j & 1) << 1)); }
 
 struct MoParams {
-#if RA_MO_TMA
-  // per output: 1-D TMA maps of the output (int32, element coordinates from
-  // its 16-B aligned base, bounded by out_cap: the copy engine clips rows past
-  // the capacity) with boxes of 256 and 32 rows; tma[o] = 0: plain stores
-  CUtensorMap tmap[RA_MAX_OUTPUTS][2];
-  int32_t omis[RA_MAX_OUTPUTS];  // rows of out[o]'s 16-B chunk before out[o]
-#endif
-  int32_t tma[RA_MAX_OUTPUTS];
   const int32_t* abase;  // 16-B aligned base, = d_in - mis
   int64_t n;
   uint32_t* hdr;
@@ -186,7 +170,7 @@ constexpr int ring_ints() {
 template <int M>
 struct __align__(128) MoSmem : MoFixed<M> {
   static constexpr int RING = ring_ints<M>();
-  alignas(128) int32_t ring[RING];  // runs start at multiples of 32 rows (128 B): TMA store sources
+  alignas(128) int32_t ring[RING];  // runs start at multiples of 32 rows (128-B aligned)
 };
 static_assert(MoSmem<1>::RING >= Cfg<1>::TILE && MoSmem<2>::RING >= 2 * Cfg<2>::TILE &&
                   MoSmem<3>::RING >= 3 * Cfg<3>::TILE && MoSmem<4>::RING >= 4 * Cfg<4>::TILE,
@@ -265,14 +249,6 @@ __device__ __forceinline__ int32_t ld_acquire_shared(const int32_t* p) {
 }
 __device__ __forceinline__ void st_release_shared(int32_t* p, int32_t v) {
   asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
-}
-// TMA bulk tensor store of one box of a 1-D int32 map: global rows
-// [x, x + box) <- shared rows at src (128-B aligned); rows past the map's
-// extent are not written.
-__device__ __forceinline__ void tma_store_1d(const CUtensorMap* map, int32_t x, const int32_t* src) {
-  asm volatile("cp.async.bulk.tensor.1d.global.shared::cta.bulk_group [%0, {%1}], [%2];" ::"l"(map), "r"(x),
-               "r"(smem_u32(src))
-               : "memory");
 }
 __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
   uint32_t v;
@@ -600,20 +576,16 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
 
   if (warp >= WR0) {
     // ========================= writers: ring -> outputs =======================
-    // RA_MO_TMA: one elected lane streams each placed run with TMA bulk tensor
-    // stores (boxes of 256 and 32 rows at element coordinates) and the warp
-    // writes the last < 32 rows.  Default: NWR writer warps copy with
-    // coalesced 128-B warp stores, WU loads in flight per lane (measured
-    // faster on B200 for dense runs: DESIGN.md §7).  Plain stores also serve
-    // outputs that cannot take a TMA map (capacity >= 2^31 rows).
+    // NWR writer warps copy each placed tile's runs, in tile order, with
+    // coalesced 128-B warp stores and WU ring loads in flight per lane.
+    // (TMA bulk tensor stores of the runs — 1-D maps, element coordinates —
+    // were measured slower for dense runs: DESIGN.md §7.)
     const int wt = tid - 32 * WR0;
     constexpr int WT = 32 * NWR, WU = RA_MO_WU;
     for (int k = 0;; ++k) {
       MWAIT(&S.placed[k % K], (uint32_t)((k / K) & 1), 4, (int)k);
       if (S.tidx[k % K] < 0) break;
       MWAIT(&S.scattered[k % K], (uint32_t)((k / K) & 1), 5, (int)k);
-      if (RA_MO_TMA && wt == 0) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // ring -> copy engine
-      if (RA_MO_TMA) __syncwarp();
       int32_t base = S.start[k % K];
       PROF_T0(t_wr);
 #pragma unroll
@@ -623,36 +595,17 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
         const int32_t* run = S.ring + base;
         int32_t* __restrict__ out = P.out[o] + g;
         const int64_t cap = P.out_cap[o] - g;  // rows of this run that fit
-#if RA_MO_TMA
-        if (P.tma[o]) {
-          const int32_t i32 = c & ~31;
-          if (wt == 0 && g < P.out_cap[o]) {
-            const int32_t G = (int32_t)(g + P.omis[o]);
-            int32_t i = 0;
-            for (; i + 256 <= c; i += 256) tma_store_1d(&P.tmap[o][0], G + i, run + i);
-            for (; i < i32; i += 32) tma_store_1d(&P.tmap[o][1], G + i, run + i);
-          }
-          const int32_t e = i32 + wt;
-          if (wt < 32 && e < c && e < cap) out[e] = run[e];
-        } else
-#endif
-        {
-          const int64_t lim = cap < 0 ? 0 : (cap > c ? c : cap);
-          int e = wt;
-          for (; e + (WU - 1) * WT < (int)lim; e += WU * WT) {
-            int32_t a[WU];
+        const int64_t lim = cap < 0 ? 0 : (cap > c ? c : cap);
+        int e = wt;
+        for (; e + (WU - 1) * WT < (int)lim; e += WU * WT) {
+          int32_t a[WU];
 #pragma unroll
-            for (int u = 0; u < WU; ++u) a[u] = run[e + u * WT];
+          for (int u = 0; u < WU; ++u) a[u] = run[e + u * WT];
 #pragma unroll
-            for (int u = 0; u < WU; ++u) out[e + u * WT] = a[u];
-          }
-          for (; e < (int)lim; e += WT) out[e] = run[e];
+          for (int u = 0; u < WU; ++u) out[e + u * WT] = a[u];
         }
+        for (; e < (int)lim; e += WT) out[e] = run[e];
         base += (c + 31) & ~31;
-      }
-      if (RA_MO_TMA && wt == 0) {
-        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // the copy engine has read the runs
       }
       writer_bar();  // every writer is done reading the ring
       PROF_ADD(16, t_wr);
@@ -662,7 +615,6 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
         mbar_arrive(&S.written[k % K]);  // release: the ring space
       }
     }
-    if (RA_MO_TMA && wt == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // outputs written
     return;
   }
 
@@ -750,11 +702,10 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
       mbar_arrive(&S.counted[i % K]);
       PROF_ADD(13, t_g0);
     }
-    if (gtid == (RA_MO_SPLIT ? 32 : 0)) {  // (RA_MO_SPLIT: another warp allocates while gtid 0 publishes)
+    if (gtid == 0) {
       int32_t rows_in = 0;
 #pragma unroll
       for (int o = 0; o < M; ++o) rows_in += (agg[o] + 31) & ~31;
-      if (RA_MO_SPLIT && i >= K) MWAIT(&S.written[i % K], (uint32_t)(((i / K) - 1) & 1), 8, (int)i);
       // ---- allocate the tile's runs, in CTA tile order (after tile i-1's).
       // Virtual ring coordinates grow monotonically; a run set that would
       // cross the physical end starts at the next multiple of RING.  Pending
@@ -861,31 +812,6 @@ size_t mo_workspace_bytes(int64_t n) {
   return ((SEL_HDR_BYTES + 16 * (size_t)tiles + 16) + 255) / 256 * 256;
 }
 
-#if RA_MO_TMA
-// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda)
-PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
-    void* f = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
-        q != cudaDriverEntryPointSuccess)
-      f = nullptr;
-    return (PFN_cuTensorMapEncodeTiled_v12000)f;
-  }();
-  return fn;
-}
-
-// 1-D int32 map over out[0 .. cap) (from its 16-B aligned base, offset mis rows)
-bool encode_out_map(CUtensorMap* map, int32_t* out, int64_t cap, int32_t mis, uint32_t box) {
-  auto enc = tensor_map_encoder();
-  if (!enc) return false;
-  cuuint64_t dim[1] = {(cuuint64_t)(cap + mis)};
-  cuuint32_t boxd[1] = {box}, estr[1] = {1};
-  return enc(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 1, (void*)(out - mis), dim, nullptr, boxd, estr,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
-#endif
 
 int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int M, int32_t* const* d_outs,
                         const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s) {
@@ -916,15 +842,6 @@ int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int
     P.out[o] = d_outs[o];
     P.out_cap[o] = out_caps[o];
     P.d_count[o] = d_counts[o];
-    // TMA stores need element coordinates (int32) below 2^31: outputs whose
-    // rows (and the input's) stay below that; others take plain stores
-    P.tma[o] = 0;
-#if RA_MO_TMA
-    P.omis[o] = (int32_t)(((uintptr_t)d_outs[o] & 15u) >> 2);
-    if (out_caps[o] > 0 && n + 64 < ((int64_t)1 << 31) && out_caps[o] + P.omis[o] < ((int64_t)1 << 31))
-      P.tma[o] = encode_out_map(&P.tmap[o][0], d_outs[o], out_caps[o], P.omis[o], 256) &&
-                 encode_out_map(&P.tmap[o][1], d_outs[o], out_caps[o], P.omis[o], 32);
-#endif
   }
   const int64_t tile = mo_tile_rows(M);
   const int64_t ntiles = n > 0 ? (n + P.mis + tile - 1) / tile : 0;

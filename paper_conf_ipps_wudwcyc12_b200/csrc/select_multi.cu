@@ -55,6 +55,11 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 #ifndef RA_MO_NWR
 #define RA_MO_NWR 4  // writer warps per CTA (aux warps fill whole warpgroups)
 #endif
+#ifndef RA_MO_NWR34
+#define RA_MO_NWR34 RA_MO_NWR  // M = 3, 4 (their dense passes are writer-bound)
+#define RA_MO_REGS34 RA_MO_REGS
+#define RA_MO_AUXREGS34 RA_MO_AUXREGS
+#endif
 #ifndef RA_MO_REGS
 // setmaxnreg: the compute warpgroups run with RA_MO_REGS registers, the aux
 // warpgroups (look-back, producer, writers) with RA_MO_AUXREGS; an increase is
@@ -81,7 +86,6 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 #define RA_MO_IN_KB 96  // input ring per CTA
 #endif
 constexpr int NG = RA_MO_NG;
-constexpr int NWR = RA_MO_NWR;
 constexpr int GW = 8;                         // warps per compute group
 constexpr int GT = 32 * GW;                   // threads per compute group
 constexpr int NCW = NG * GW;                  // compute warps
@@ -90,7 +94,6 @@ constexpr int NCW = NG * GW;                  // compute warps
 #endif
 constexpr int NLB = RA_MO_NLB;
 constexpr int LBWARP = NCW, PRWARP = NCW + NLB, WR0 = NCW + NLB + 1;
-constexpr int BLOCK = 32 * (NCW + NLB + 1 + NWR);
 #ifndef RA_MO_K
 #define RA_MO_K 8
 #endif
@@ -115,6 +118,10 @@ struct Cfg {
   static constexpr int W = (M + 1) / 2;              // status words per tile
   static constexpr int INSLOTS = (M <= 2 ? RA_MO_IN_KB : RA_MO_IN_KB34) * 1024 / (TILE * 4);
   static constexpr int D1 = RA_MO_D1 > 0 ? RA_MO_D1 : (M == 1 ? 2 : 1);
+  static constexpr int NWR = M <= 2 ? RA_MO_NWR : RA_MO_NWR34;           // writer warps
+  static constexpr int BLOCK = 32 * (NCW + NLB + 1 + NWR);
+  static constexpr int REGS = M <= 2 ? RA_MO_REGS : RA_MO_REGS34;         // setmaxnreg: compute warps
+  static constexpr int AUXREGS = M <= 2 ? RA_MO_AUXREGS : RA_MO_AUXREGS34;  // and aux warps
 };
 __host__ __device__ constexpr int q_of(int npk, int j) { return npk == 2 ? (j & 1) : 0; }
 __host__ __device__ constexpr int b_of(int npk, int j) { return npk == 2 ? (j >> 1) : ((j >> 1) | ((j & 1) << 1)); }
@@ -261,6 +268,7 @@ __device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
 __device__ __forceinline__ void group_bar(int g) {  // named barriers 1..NG: one compute group
   asm volatile("bar.sync %0, %1;" ::"r"(1 + g), "n"(GT) : "memory");
 }
+template <int NWR>
 __device__ __forceinline__ void writer_bar() {
   asm volatile("bar.sync %0, %1;" ::"n"(1 + NG), "n"(32 * NWR) : "memory");
 }
@@ -384,7 +392,7 @@ __device__ __forceinline__ void window_sums(const MoSmem<M>& S, const MoParams& 
 }
 
 template <int M, bool HAS_NE>
-__global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_constant__ MoParams P) {
+__global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __grid_constant__ MoParams P) {
   using C = Cfg<M>;
   using SM = MoSmem<M>;
   constexpr int TILE = C::TILE, VEC = C::VEC, NPK = C::NPK, W = C::W, INSLOTS = C::INSLOTS, D1 = C::D1;
@@ -428,8 +436,8 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
   // register file is rebalanced: compute warpgroups get more registers, the
   // latency-bound aux warpgroups fewer (setmaxnreg, whole warpgroups).
 #if RA_MO_REGS
-  static_assert(NCW % 4 == 0 && (BLOCK / 32) % 4 == 0, "setmaxnreg works on whole warpgroups");
-  if (warp >= NCW) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(RA_MO_AUXREGS));
+  static_assert(NCW % 4 == 0 && (C::BLOCK / 32) % 4 == 0, "setmaxnreg works on whole warpgroups");
+  if (warp >= NCW) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::AUXREGS));
 #endif
   if (warp == PRWARP) {
     // ========================= producer: partition + load =====================
@@ -581,7 +589,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
     // (TMA bulk tensor stores of the runs — 1-D maps, element coordinates —
     // were measured slower for dense runs: DESIGN.md §7.)
     const int wt = tid - 32 * WR0;
-    constexpr int WT = 32 * NWR, WU = RA_MO_WU;
+    constexpr int NWR = C::NWR, WT = 32 * NWR, WU = RA_MO_WU;
     for (int k = 0;; ++k) {
       MWAIT(&S.placed[k % K], (uint32_t)((k / K) & 1), 4, (int)k);
       if (S.tidx[k % K] < 0) break;
@@ -607,7 +615,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
         for (; e < (int)lim; e += WT) out[e] = run[e];
         base += (c + 31) & ~31;
       }
-      writer_bar();  // every writer is done reading the ring
+      writer_bar<NWR>();  // every writer is done reading the ring
       PROF_ADD(16, t_wr);
       if (wt == 0) {
         PROF_LAT(19, S.t_placed[k % K]);
@@ -620,7 +628,7 @@ __global__ void __launch_bounds__(BLOCK, 1) select_multi_kernel(const __grid_con
 
   // ========================= compute groups =====================================
 #if RA_MO_REGS
-  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(RA_MO_REGS));
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REGS));
 #endif
   const int g = warp / GW, wg = warp % GW, gtid = tid - GT * g;
   for (int i = g;; i += NG) {
@@ -794,7 +802,7 @@ int launch_mo(const MoParams& P, int64_t ntiles, cudaStream_t s) {
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
   if (grid > ntiles) grid = ntiles;
   if (grid < 1) grid = 1;
-  cudaError_t e = launch_pdl(select_multi_kernel<M, HAS_NE>, dim3((unsigned)grid), dim3(BLOCK), sizeof(MoSmem<M>), s, P);
+  cudaError_t e = launch_pdl(select_multi_kernel<M, HAS_NE>, dim3((unsigned)grid), dim3(Cfg<M>::BLOCK), sizeof(MoSmem<M>), s, P);
   count_launch();
   if (e != cudaSuccess) return cuda_fail(e, "select_multi_kernel launch");
   return RA_OK;

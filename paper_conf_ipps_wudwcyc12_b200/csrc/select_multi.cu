@@ -1,37 +1,37 @@
-// select_multi.cu — several SELECTs filtering the same input in ONE pass
-// (SURVEY §8(f) f2): "different SELECT operators need to filter the same input
-// data" (Fig 2(c)).  Output o is the order-preserving SELECT
-// of the input by predicate chain o, o < M <= RA_MAX_OUTPUTS (4).
+// select_multi.cu — SELECT as one warp-specialised pass for sm_100a: the
+// fused chain (one output) and several SELECTs filtering the same input
+// ("different SELECT operators need to filter the same input
+// data", Fig 2(c)).  Output o is the order-preserving
+// SELECT of the input by predicate chain o, o < M <= RA_MAX_OUTPUTS (4).
 //
 // The input is read once; every output has its own compaction and its own
 // global offsets.  The paper's four stages (partition, filter, buffer, gather;
 // Fig 3) are split over specialised warps of one
-// persistent CTA per SM:
+// persistent 768-thread CTA per SM:
 //
-//   producer warp   draws tiles by atomic ticket, bulk-copies each (TMA engine)
-//                   into a ring of input slots (96 KB in flight per SM)
-//   compute groups  NG groups of 8 warps take alternate tiles: filter (all M
-//                   folded predicates in registers), per-output warp counts,
-//                   publish the M tile aggregates, then compact each output's
-//                   matches into a shared-memory ring of selected rows
-//   look-back warp  decoupled look-back over the published aggregates: each
-//                   tile's M global offsets
-//   writer warps    copy each placed tile's M runs from the ring to the
-//                   outputs, in tile order, with coalesced stores
+//   producer warp    draws tiles by atomic ticket, bulk-copies each 32 KB tile
+//                    (TMA engine) into a ring of input slots
+//   2 compute groups 8 warps each, alternate tiles: filter (all M folded
+//                    predicates in registers), per-output warp counts, publish
+//                    the M tile aggregates at once, allocate the tile's runs in
+//                    a shared ring of selected rows (in tile order), compact
+//                    each output's matches into its run
+//   3 look-back warps decoupled look-back over the published aggregates: warp
+//                    r resolves tiles r, r+3, ... (bulk-copied windows of status
+//                    words, branch-free sums), prefixes chained in shared memory
+//   4 writer warps   copy each placed tile's M runs from the ring to the
+//                    outputs, in tile order, with coalesced stores
 //
-// Why writer warps (round 1's two-output kernel wrote from the compute warps):
-// when both outputs keep most rows, a tile's runs outgrow a 40 KB ring, so the
-// compute warps waited for a placement (an L2 round trip under load) or spilled
-// a run to global memory and read it back at L2 latency; measured 0.32 of the
-// copy peak at (0.9, 0.9).  Here the compute path never waits for a placement
-// except when the ring (121 KB per SM, sized so that a whole tile's M runs
-// always fit an empty ring) is full, and then only for OLDER tiles.
-//
-// Tiles are 8192 rows for M <= 2 and 4096 rows for M = 3, 4 (so M runs of a
-// tile fit the ring).  Status words: W = ceil(M/2) u64 words per tile, each
-// [flag:2 | 28-bit launch tag | two 16-bit aggregates]; a word is ready when
-// its high half carries this launch's tag, so no per-call memset (select_fused
-// uses the same scheme; see there for the look-back's lag and windows).
+// The compute path never waits for a placement (an L2 round trip under load)
+// except when the ring is full, and then only for OLDER tiles: the ring always
+// holds a whole tile's M runs.  setmaxnreg gives the compute warpgroups 88
+// registers and the latency-bound aux warpgroups 56.  Tiles are 8192 rows.
+// Status words: W = ceil(M/2) u64 words per tile, each [flag:2 | 28-bit launch
+// tag | two 16-bit aggregates]; a word is ready when its high half carries this
+// launch's tag, so no per-call memset (the launch before the tag wraps clears
+// every status word the workspace has carried).  How this design was measured
+// into shape (round 1's compute-warp writes and global spills, one look-back
+// warp, branchy window sums): DESIGN.md §7.
 
 #include <stdio.h>
 #include <stdlib.h>

@@ -136,3 +136,46 @@ def test_finalize_128bit_charge_and_domain():
     assert rc == R.RA_E_DOMAIN
     assert got[0]["sum_charge"] == 2**64 and got[0]["count_order"] == 6
     assert (got[0]["returnflag"], got[0]["linestatus"]) == ("N", "O")
+
+
+def _multi_args(M, n=100, outs=None, caps=None, cnts=None, ks=None, chains=None, ws=256, wsb=1 << 20, d_in=4096):
+    import ctypes
+    keep = [R.make_preds([("lt", 0)]) for _ in range(max(1, M))]
+    ch = (ctypes.c_void_p * max(1, M))(*(chains if chains is not None else [ctypes.addressof(p) for p in keep]))
+    k = (ctypes.c_int * max(1, M))(*(ks if ks is not None else [1] * M))
+    op = (ctypes.c_void_p * max(1, M))(*(outs if outs is not None else [8192] * M))
+    cp = (ctypes.c_int64 * max(1, M))(*(caps if caps is not None else [n] * M))
+    cn = (ctypes.c_void_p * max(1, M))(*(cnts if cnts is not None else [16384 + 8 * o for o in range(M)]))
+    return (d_in, n, ch, k, M, op, cp, cn, ws, wsb, 0), keep
+
+
+@pytest.mark.parametrize("case", ["M0", "M5", "null_ws", "misaligned_in", "misaligned_out", "misaligned_count",
+                                  "negative_cap", "k9", "bad_op", "null_chain", "small_ws", "huge_n"])
+def test_select_multi_argument_errors_without_gpu(case):
+    """ra_select_multi rejects bad arguments before touching CUDA."""
+    kw = {"M0": dict(M=0), "M5": dict(M=5), "null_ws": dict(M=2, ws=0), "misaligned_in": dict(M=2, d_in=4098),
+          "misaligned_out": dict(M=2, outs=[8192, 8194]), "misaligned_count": dict(M=2, cnts=[16384, 16388]),
+          "negative_cap": dict(M=2, caps=[10, -1]), "k9": dict(M=1, ks=[9]), "null_chain": dict(M=2, chains=[0, 0]),
+          "small_ws": dict(M=3, n=1 << 24, wsb=4096), "huge_n": dict(M=1, n=1 << 34, wsb=1 << 40)}
+    if case == "bad_op":
+        import ctypes
+        bad = R.make_preds([(17, 0)])
+        args, keep = _multi_args(1, chains=[ctypes.addressof(bad)])
+    else:
+        args, keep = _multi_args(**kw[case])
+    with pytest.raises(R.RAError) as e:
+        R.ra_select_multi(*args)
+    assert e.value.code == (R.RA_E_WORKSPACE if case == "small_ws" else R.RA_E_INVAL), (case, R.ra_last_error())
+
+
+def test_select_offsets_argument_errors_without_gpu():
+    for bad in (0, -3, R.RA_MAX_RANKS + 1):
+        with pytest.raises(R.RAError) as e:
+            R.ra_select_offsets(4096, bad, 8192, 16384, 0)
+        assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:  # no output at all
+        R.ra_select_offsets(4096, 4, 0, 0, 0)
+    assert e.value.code == R.RA_E_INVAL
+    with pytest.raises(R.RAError) as e:  # misaligned
+        R.ra_select_offsets(4100, 4, 8192, 0, 0)
+    assert e.value.code == R.RA_E_INVAL

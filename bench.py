@@ -463,6 +463,18 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
                          "fused_over_unfused": ums / chain_ms, "launches_per_step": k}
         del uo, uws
 
+    # --- library yardstick: the same chain as PyTorch ops
+    # (elementwise compares -> mask -> torch.masked_select); not our path
+    def torch_chain(i=0, kernel_done=False):
+        m = x < preds[0][1]
+        for _, t in preds[1:]:
+            m &= x < t
+        return torch.masked_select(x, m)
+    assert torch_chain().numel() == kept
+    tms_, _ = timed(torch, D, torch_chain, 10, 3)
+    ex["yardstick_torch_masked_select"] = {"ms_per_step": tms_, "ours_speedup": tms_ / chain_ms,
+                                           "ops": "x < T_j (k compares, &=) then torch.masked_select"}
+
     # --- e2e: same chain from pinned host memory through ra_fission_run
     if True:  # every rank streams its own shard from pinned host memory
         h_in = torch.empty(n, dtype=torch.int32, pin_memory=True)

@@ -220,21 +220,23 @@ def test_unfused_workspace_larger_than_required(R, extra):
     np.testing.assert_array_equal(out[:exp.size].cpu().numpy(), exp)
 
 
-def test_epoch_tag_wrap_clears_stale_status_words(R):
+@pytest.mark.parametrize("base", [0, 1 << 21], ids=["single_output_kernel", "multi_output_pass"])
+def test_epoch_tag_wrap_clears_stale_status_words(R, base):
     """Status words carry a 28-bit launch tag.  A word left by a launch exactly
     2^28 launches earlier carries the tag the wrapped epoch will use again: the
     launch before the wrap must clear every word the workspace has held (header
     high-water mark), so a later, larger launch never reads such a word as a
     published aggregate.  Simulated by planting the header and stale words."""
-    n_small, n_big = 5 * 8192 + 11, 40 * 8192 + 5
+    n_small, n_big = base + 5 * 8192 + 11, base + 40 * 8192 + 5
+    hw = (n_big + 8191) // 8192 + 7  # words carried so far: more than the big launch's tiles
     ws = torch.zeros(R.ra_select_workspace_bytes(n_big, 1, 1), dtype=torch.uint8, device="cuda")
     words = ws[256:].view(torch.int64)
     hdr32, hdr64 = ws[:256].view(torch.int32), ws[:256].view(torch.int64)
     flag_a, tag_shift = 1 << 62, 34
     # stale words of "tag 0" (a launch 2^28 launches ago) with bogus aggregates
-    words[:48] = flag_a | (0 << tag_shift) | 1000
+    words[:hw] = flag_a | (0 << tag_shift) | 1000
     hdr32[0] = (1 << 28) - 1      # this launch uses the last tag before the wrap
-    hdr64[3] = 48                 # high-water mark: 48 words carried so far
+    hdr64[3] = hw                 # high-water mark: hw words carried so far
     preds = [("lt", 0)]
     sh = int(torch.cuda.current_stream().cuda_stream)
     P = R.make_preds(preds)
@@ -247,7 +249,7 @@ def test_epoch_tag_wrap_clears_stale_status_words(R):
         exp = oracle.select(x.cpu().numpy(), preds)
         assert int(cnt.item()) == exp.size, n
         np.testing.assert_array_equal(out[:exp.size].cpu().numpy(), exp)
-    assert int(hdr32[0].item()) == (1 << 28) + 2 and int(hdr64[3].item()) == 48
+    assert int(hdr32[0].item()) == (1 << 28) + 2 and int(hdr64[3].item()) == hw
 
 
 def test_select_rows_workspace_reuse_across_sizes(R):
@@ -267,3 +269,39 @@ def test_select_rows_workspace_reuse_across_sizes(R):
         assert c == exp_ids.size
         np.testing.assert_array_equal(ids[:c].cpu().numpy().astype(np.int64), exp_ids)
         np.testing.assert_array_equal(outs[0][:c].cpu().numpy(), pay[exp_ids])
+
+
+def test_one_workspace_across_both_pass_kinds(R):
+    """The fused chain runs the single-output kernel up to 2^21 rows and the
+    multi-output pass above (same header, same one-word-per-8192-row status
+    format): one workspace alternating between them, sizes on both sides of
+    the threshold, every result exact."""
+    sizes = [(1 << 21) - 7, (1 << 21) + 9, 1 << 20, 3 << 21, 12345, (1 << 22) + 1, 1 << 21, 5, (1 << 21) + 1]
+    ws_b = R.ra_select_workspace_bytes(max(sizes), 2, 1)
+    ws = torch.zeros(ws_b, dtype=torch.uint8, device="cuda")
+    sh = int(torch.cuda.current_stream().cuda_stream)
+    for i, n in enumerate(sizes):
+        x = torch.from_numpy(ragen.int32_column(500 + i, n)).cuda()
+        preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 2)]
+        out = torch.empty(n, dtype=torch.int32, device="cuda")
+        cnt = torch.empty(1, dtype=torch.int64, device="cuda")
+        R.ra_select_chain(x.data_ptr(), n, R.make_preds(preds), 2, 1, out.data_ptr(), n, cnt.data_ptr(),
+                          ws.data_ptr(), ws_b, sh)
+        torch.cuda.synchronize()
+        exp = oracle.select(x.cpu().numpy(), preds)
+        assert int(cnt.item()) == exp.size, (i, n)
+        np.testing.assert_array_equal(out[:exp.size].cpu().numpy(), exp)
+
+
+@pytest.mark.parametrize("s", [0.01, 0.25, 0.5, 0.9])
+@pytest.mark.parametrize("k", [1, 3])
+def test_chain_sweep_multi_output_pass(R, s, k):
+    """The selectivity sweep above 2^21 rows (the fused chain's warp-specialised
+    pass), with a misaligned start and a ragged tail."""
+    n = (1 << 22) + 777
+    x = ragen.int32_column(3, n)
+    preds = [("lt", t) for t in ragen.nested_thresholds(s, k)]
+    exp = oracle.select(x, preds)
+    got, c = run(R, x, preds, offset=1)
+    assert c == exp.size
+    np.testing.assert_array_equal(got[:c], exp)

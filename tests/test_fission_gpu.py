@@ -92,3 +92,18 @@ def test_full_size_config_3_host_resident_2_pow_30(R, streams):
     exp = oracle.select(h.numpy(), preds)
     assert c == exp.size
     np.testing.assert_array_equal(h_out.numpy()[:c], exp)
+
+
+@pytest.mark.parametrize("chunk", [(1 << 22) + 5, (1 << 21) + 1, 3 << 20])
+@pytest.mark.parametrize("nstreams", [1, 3])
+def test_fission_chunks_above_the_small_pass_threshold(R, streams, chunk, nstreams):
+    """Chunks above 2^21 rows run the multi-output pass per chunk, smaller
+    trailing chunks the single-output kernel: ragged chunking over 5M rows,
+    equal to the oracle."""
+    n = 5_000_003
+    x = ragen.int32_column(90, n)
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.5, 2)]
+    exp = oracle.select(x, preds)
+    h_out, c = R.fission_run(pinned(x), preds, chunk, streams[:nstreams])
+    assert c == exp.size
+    assert np.array_equal(h_out[:c].numpy(), exp)

@@ -121,8 +121,10 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
 
 // Several SELECTs on one input in one pass (select_multi.cu), 1 <= M <= 4:
 // cp[o] = output o's folded chain; validated arguments.
+// d_n (nullable): device-resident row count (<= n) of the input, from a previous pass.
 int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int M, int32_t* const* d_outs,
-                        const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s);
+                        const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s,
+                        const int64_t* d_n = nullptr);
 size_t mo_workspace_bytes(int64_t n);
 
 // Payload fields of a tuple SELECT.  The selectivity decides, on the device,

@@ -1,9 +1,10 @@
 // select_fused.cu — single-pass, single-output SELECT for sm_100a: the
-// passes of the unfused chain ("without round trip", one predicate per pass,
-// row count from the previous pass on the device) and the tuple SELECT's key
-// pass (row ids + order masks for the payload compaction).  The fused chain
-// and several SELECTs on one input run select_multi.cu's warp-specialised
-// pass (writer warps, cooperative look-back), measured faster on B200.
+// tuple SELECT's key pass (row ids + order masks for the payload compaction)
+// and every SELECT pass over at most 2^21 rows (fused chain or one pass of the
+// unfused chain), where its lighter launch wins.  Larger fused chains, the
+// unfused chain's larger passes and several SELECTs on one input run
+// select_multi.cu's warp-specialised pass (writer warps, cooperative
+// look-back), measured faster on B200.
 //
 // The paper's SELECT has four stages — partition, filter, buffer, gather —
 // in two CUDA kernels separated by a global synchronisation so that each CTA
@@ -804,6 +805,8 @@ int launch_select_pass(const int32_t* d_in, int64_t n_max, const int64_t* d_n, c
 int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, int k, int fused,
                       int32_t* d_out, int64_t out_cap, int64_t* d_count, void* d_ws,
                       size_t ws_bytes, cudaStream_t s) {
+  static const int64_t small_rows =
+      getenv("RA_SEL_SMALL_ROWS") ? atoll(getenv("RA_SEL_SMALL_ROWS")) : RA_SEL_SMALL_ROWS_DEFAULT;
   if (fused || k <= 1) {
     // the fused chain is one output of the warp-specialised multi-output pass
     // (select_multi.cu): one kernel, writer warps, cooperative look-back.
@@ -811,8 +814,6 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
     // single-output kernel of this file starts faster there (both produce the
     // same result; same workspace layout for one output).  RA_SEL_SMALL_ROWS
     // (diagnostics) moves the threshold.
-    static const int64_t small_rows =
-        getenv("RA_SEL_SMALL_ROWS") ? atoll(getenv("RA_SEL_SMALL_ROWS")) : RA_SEL_SMALL_ROWS_DEFAULT;
     CanonPred cp;
     int rc = canonicalize(h_preds, k, &cp);
     if (rc) return rc;
@@ -835,7 +836,12 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
     const bool last = (j == k - 1);
     int32_t* dst = last ? d_out : buf[j & 1];
     int64_t* dcnt = last ? d_count : &cnt[j & 1];
-    rc = launch_select_pass(src, n, src_n, cp, dst, last ? out_cap : n, dcnt, d_ws, s, nullptr);
+    // each pass is the same SELECT machinery as the fused chain (the
+    // multi-output pass above the small-input threshold), so the fused /
+    // unfused comparison measures fusion, not two kernel designs
+    int64_t cap = last ? out_cap : n;
+    rc = n <= small_rows ? launch_select_pass(src, n, src_n, cp, dst, cap, dcnt, d_ws, s, nullptr)
+                         : launch_select_multi(src, n, &cp, 1, &dst, &cap, &dcnt, d_ws, s, src_n);
     if (rc) return rc;
     src = dst;
     src_n = dcnt;

@@ -128,7 +128,8 @@ __host__ __device__ constexpr int b_of(int npk, int j) { return npk == 2 ? (j >>
 
 struct MoParams {
   const int32_t* abase;  // 16-B aligned base, = d_in - mis
-  int64_t n;
+  int64_t n;             // rows (host bound)
+  const int64_t* d_n;    // optional device row count (<= n): the previous pass's count (unfused chain)
   uint32_t* hdr;
   unsigned long long* ticket;
   uint64_t* status;      // status[tile * W + j]
@@ -403,7 +404,12 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
 
   dev::grid_dep_wait();  // programmatic dependent launch: previous grid's writes visible
   if (tid == 0) {
-    S.n = P.n;
+    int64_t n = P.n;
+    if (P.d_n) {
+      const int64_t dn = dev::ld_relaxed_s64(P.d_n);
+      n = dn < n ? (dn < 0 ? 0 : dn) : n;
+    }
+    S.n = n;
     S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);
     S.demand = -1;
     S.a_va = 0;
@@ -822,7 +828,8 @@ size_t mo_workspace_bytes(int64_t n) {
 
 
 int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int M, int32_t* const* d_outs,
-                        const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s) {
+                        const int64_t* out_caps, int64_t* const* d_counts, void* d_ws, cudaStream_t s,
+                        const int64_t* d_n) {
   if (M < 1 || M > RA_MAX_OUTPUTS) return fail(RA_E_INVAL, "M=%d outside [1, %d]", M, RA_MAX_OUTPUTS);
   if (n >= ((int64_t)1 << 34)) return fail(RA_E_INVAL, "n=%lld >= 2^34", (long long)n);
   MoParams P;
@@ -831,6 +838,7 @@ int launch_select_multi(const int32_t* d_in, int64_t n, const CanonPred* cp, int
   P.mis = (int32_t)((a & 15u) >> 2);
   P.abase = (const int32_t*)(a - (a & 15u));
   P.n = n;
+  P.d_n = d_n;
   P.hdr = (uint32_t*)d_ws;
   P.ticket = (unsigned long long*)((char*)d_ws + 8);
   P.status = (uint64_t*)((char*)d_ws + SEL_HDR_BYTES);

@@ -1,4 +1,3 @@
 mkdir -p gpurun_out
-for v in w8wd w8bwd; do RA_LIB_PATH=$PWD/build/libra_$v.so timeout -s KILL 300 python -m pytest tests/test_select_multi_gpu.py -x -q -p no:cacheprovider -k "three_four or many_outputs" 2>&1 | tail -1; done
-( timeout -s KILL 120 python scripts/mo_quick.py
-  for v in w8 w8b; do RA_LIB_PATH=$PWD/build/libra_$v.so timeout -s KILL 120 python scripts/mo_quick.py; done ) 2>&1 | tee gpurun_out/mo_variants18.txt
+RA_LIB_PATH=$PWD/build/libra_wd.so timeout -s KILL 600 python -m pytest tests/test_select_gpu.py tests/test_fission_gpu.py -x -q -p no:cacheprovider -k "not 2_pow_31" 2>&1 | tail -1
+timeout -s KILL 600 python scripts/sweeps.py d2 gpurun_out/d2_sweep.txt; echo d2 rc=$?

@@ -26,8 +26,6 @@ CAPTURES = {  # report -> (summary name, traffic key, command)
                         "python scripts/prof_driver.py select 5 28 1 0.01  (2^28 int32, k=1, s=0.01; select_multi_kernel<1>)"),
     "prof_select_s09": ("select_chain_k1_s09_n28", "select_chain_k1_s0.9_n28",
                         "python scripts/prof_driver.py select 5 28 1 0.9  (2^28 int32, k=1, s=0.9; select_multi_kernel<1>)"),
-    "prof_unfused": ("unfused_pass_k2_s05_n28", "unfused_pass_k2_s0.5_n28",
-                     "python scripts/prof_driver.py unfused 5  (first pass of the unfused chain: select_fused_kernel)"),
     "prof_q1": ("q1_sf10", "q1_sf10", "python scripts/prof_driver.py q1 5  (SF10, 60M rows)"),
     "prof_rows": ("select_rows_k2_s05_n28", "select_rows_k2_s0.5_n28",
                   "python scripts/prof_driver.py rows 5  (2^28 key + 2 int32 fields, k=2, s=0.5/stage)"),

@@ -18,7 +18,7 @@ bd = torch.from_numpy(base).cuda()
 fstreams = [torch.cuda.Stream() for _ in range(3)]
 t0 = time.time()
 for it in range(iters):
-    n = int(rng.choice([0, 1, 7, 4096, 8192, 8193, 100_003, 1 << 20, (1 << 22) - 5]))
+    n = int(rng.choice([0, 1, 7, 4096, 8192, 8193, 100_003, 1 << 20, (1 << 21) + 3, (1 << 22) - 5]))
     off = int(rng.integers(0, 4))
     x, xd = base[off:off + n], bd[off:off + n]
     t = int(rng.integers(-2**31, 2**31 - 1))
@@ -28,13 +28,15 @@ for it in range(iters):
         e = x[(x < t) & (x != 5)]
         c = int(c.item())
         assert c == e.size and np.array_equal(out[:c].cpu().numpy(), e), ("chain", it, n, off, t)
-    elif kind == 1:
-        t2 = int(rng.integers(-2**31, 2**31 - 1))
-        outs, cnt = R.select_multi(xd, [[("lt", t)], [("gt", t2)]])
-        e0, e1 = x[x < t], x[x > t2]
-        c0, c1 = (int(v) for v in cnt.cpu().tolist())
-        assert c0 == e0.size and c1 == e1.size, ("multi", it, n, off)
-        assert np.array_equal(outs[0][:c0].cpu().numpy(), e0) and np.array_equal(outs[1][:c1].cpu().numpy(), e1)
+    elif kind == 1:  # 1..4 SELECTs on one input, alternating < and > thresholds
+        M = int(rng.integers(1, 5))
+        ts = [int(rng.integers(-2**31, 2**31 - 1)) for _ in range(M)]
+        chains = [[("lt", ts[o])] if o % 2 == 0 else [("gt", ts[o])] for o in range(M)]
+        outs, cnt = R.select_multi(xd, chains)
+        cs = [int(v) for v in cnt.cpu().tolist()][:M]
+        for o in range(M):
+            e = x[x < ts[o]] if o % 2 == 0 else x[x > ts[o]]
+            assert cs[o] == e.size and np.array_equal(outs[o][:cs[o]].cpu().numpy(), e), ("multi", it, n, off, M, o)
     elif kind == 2:
         ids, outs, c = R.select_rows(xd, [("lt", t)], [xd], rowids=bool(rng.integers(0, 2)))
         e = x[x < t]

@@ -233,6 +233,10 @@ RA_API size_t ra_select_rows_workspace_bytes(int64_t n, int k) {
          (((size_t)n * 4 + 255) / 256) * 256;
 }
 
+#ifndef RA_TUPLE_STAGE_DEN
+#define RA_TUPLE_STAGE_DEN 32  // without caller ids the key pass stages the first n/32 (A/B knob)
+#endif
+
 RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_preds, int k, uint32_t* d_rowids,
                           const ra_payload* h_payloads, int m, int64_t out_cap, int64_t* d_count, void* d_ws,
                           size_t ws_bytes, ra_stream_t stream) {
@@ -253,7 +257,7 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   GatherSpec g;
   g.m = m;
   g.n = n;
-  g.sparse_den = 32;  // 4-byte fields: gather below 1/32 selected (measured crossover)
+  g.sparse_den = 10;  // 4-byte fields: gather up to 1/10 selected (measured crossover)
   for (int j = 0; j < m; ++j) {
     const ra_payload& p = h_payloads[j];
     if (p.elem_bytes != 4 && p.elem_bytes != 8)
@@ -264,11 +268,15 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
     g.elem_bytes[j] = p.elem_bytes;
     g.col[j] = p.col;
     g.out[j] = p.out;
-    if (p.elem_bytes == 8) g.sparse_den = 8;  // 8-byte fields: sectors hold 4 rows, gather pays longer
+    if (p.elem_bytes == 8) g.sparse_den = 4;  // 8-byte fields: one gathered row moves 2x the bytes, crossover 1/4
   }
   CanonPred cp;
   rc = canonicalize(h_preds, k, &cp);
   if (rc) return rc;
+  // Without caller ids the ids of the sparse path come from the key pass (the
+  // first n/32, staged) and ids_kernel (the rest, from the order masks): the
+  // crossover with the compaction is at a lower selectivity.
+  if (!d_rowids) g.sparse_den = g.sparse_den == 4 ? 8 : 12;
   if (getenv("RA_TUPLE_GATHER")) g.sparse_den = 0;  // A/B only: always the id gather
   // One fused pass over the key writes the caller's row ids (if asked for) and
   // the per-tile order masks; then the payload fields are placed by the gather
@@ -281,19 +289,22 @@ RA_API int ra_select_rows(const int32_t* d_key, int64_t n, const ra_pred* h_pred
   const size_t mask_off = (ws_bytes & ~(size_t)255) - extra;
   const size_t stage_off = mask_off + ((ra::sel_masks_bytes(n) + 255) / 256) * 256;
   uint32_t* ids = d_rowids ? d_rowids : (uint32_t*)((char*)d_ws + stage_off);
-  const int64_t cap = d_rowids ? out_cap : (out_cap < n ? out_cap : n);
   const int64_t T = ra::sel_max_tiles(n);
   char* mb = (char*)d_ws + mask_off;
   ra::SelMasks mk;
   mk.fmask = (uint32_t*)mb;
   mk.meta = (uint32_t*)(mb + (((size_t)T * SEL_THREADS * 4 + 255) / 256) * 256);
   const bool masks = m > 0 && g.sparse_den > 0;
-  const bool stage = !d_rowids && !masks;  // A/B: ids staged by the key pass
+  // Staging ids in the key pass costs a dense call ~0.15 ms per n of ids (the
+  // ring of selected rows fills and waits for the look-back), so only the
+  // first n/32 are staged; a count up to that needs no ids_kernel at all.
+  int64_t cap = d_rowids ? out_cap : (out_cap < n ? out_cap : n);
+  if (!d_rowids && masks && cap > n / RA_TUPLE_STAGE_DEN) cap = n / RA_TUPLE_STAGE_DEN;
   rc = launch_select_pass(d_key, n, nullptr, cp, nullptr, cap, d_count, d_ws, (cudaStream_t)stream,
-                          (d_rowids && cap > 0) || stage ? ids : nullptr, masks ? &mk : nullptr);
+                          (d_rowids || m > 0) && cap > 0 ? ids : nullptr, masks ? &mk : nullptr);
   if (rc) return rc;
   if (masks && !d_rowids) {
-    rc = ra::launch_ids_from_masks(d_key, n, mk, d_count, g.sparse_den, ids, (cudaStream_t)stream);
+    rc = ra::launch_ids_from_masks(d_key, n, mk, d_count, g.sparse_den, cap, ids, (cudaStream_t)stream);
     if (rc) return rc;
   }
   rc = launch_gather(ids, d_count, out_cap < n ? out_cap : n, g, (cudaStream_t)stream);

@@ -243,10 +243,11 @@ __global__ void __launch_bounds__(CT_BLOCK, 2) compact_kernel(const CompactParam
 // tuple, from the order masks (one warp per 1024-row slice; predicated stores).
 __global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ fmask, const uint32_t* __restrict__ meta,
                                                   const int64_t* __restrict__ d_count, int64_t n, int32_t mis,
-                                                  int32_t sparse_den, uint32_t* __restrict__ ids) {
+                                                  int32_t sparse_den, int64_t staged, uint32_t* __restrict__ ids) {
   dev::grid_dep_wait();
   const int64_t cnt = *d_count;
   if (cnt * sparse_den > n) return;  // dense: compact_kernel places the fields, no ids needed
+  if (cnt <= staged) return;         // the key pass staged them all
   const int lane = threadIdx.x & 31;
   const int64_t nslices = (n + mis + CT_SLICE - 1) / CT_SLICE;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
@@ -266,18 +267,27 @@ __global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ f
     }
 #pragma unroll
     for (int q = 0; q < U; ++q) {
-      if (!__any_sync(0xffffffffu, fl[q] != 0u)) continue;
+      // a slice that ends before `staged` holds only ids the key pass wrote
+      // (rewriting one it did write stores the same value)
+      if (dst0[q] + CT_SLICE <= staged || !__any_sync(0xffffffffu, fl[q] != 0u)) continue;
       uint32_t ex[2], tot[2];
       packed_scan(fl[q], lane, ex, tot);
       const uint32_t r0 = (uint32_t)((sb + q) * CT_SLICE - mis);  // row of the slice's first virtual row (mod 2^32)
       uint32_t* a0 = ids + dst0[q];
-      int32_t rb = 0;
-#pragma unroll
-      for (int j = 0; j < SEL_VEC; ++j) {  // sparse: visit the set bits only
-        uint32_t* a = a0 + rb + ((ex[j & 1] >> (8 * (j >> 1))) & 0xFFu);
-        for (uint32_t nib = (fl[q] >> (4 * j)) & 0xFu; nib; nib &= nib - 1u)
-          *a++ = r0 + 4 * (32 * j + lane) + (__ffs(nib) - 1);
-        rb += (int32_t)((tot[j & 1] >> (8 * (j >> 1))) & 0xFFu);
+      // one iteration per set bit b = 4j + c of the lane (the warp runs max
+      // popcount iterations, ~1-3 on this sparse path; measured 1.5x faster
+      // than a loop over the 8 vectors and their nibbles): its position is
+      //   (warp's count in vectors j' < j) + (lanes < this one in vector j)
+      //   + (this lane's bits below c in vector j)
+      // the first term summed from the packed byte counts with dp4a.
+      for (uint32_t f = fl[q]; f; f &= f - 1u) {
+        const int b = __ffs(f) - 1, j = b >> 2;
+        const uint32_t me = (uint32_t)((1ull << (8 * ((j + 1) >> 1))) - 1u);  // even j' < j: bytes [0, ceil(j/2))
+        const uint32_t mo = (1u << (8 * (j >> 1))) - 1u;                       // odd j' < j: bytes [0, floor(j/2))
+        const uint32_t pos = __dp4a(tot[0] & me, 0x01010101u, 0u) + __dp4a(tot[1] & mo, 0x01010101u, 0u) +
+                             ((ex[j & 1] >> (8 * (j >> 1))) & 0xFFu) +
+                             __popc(fl[q] & (0xFu << (4 * j)) & ((1u << b) - 1u));
+        a0[pos] = r0 + 4 * (32 * j + lane) + (b & 3);
       }
     }
   }
@@ -286,7 +296,7 @@ __global__ void __launch_bounds__(256) ids_kernel(const uint32_t* __restrict__ f
 }  // namespace
 
 int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count,
-                          int32_t sparse_den, uint32_t* ids, cudaStream_t s) {
+                          int32_t sparse_den, int64_t staged, uint32_t* ids, cudaStream_t s) {
   if (n == 0) return RA_OK;
   const int32_t mis = (int32_t)(((uintptr_t)d_key & 15u) >> 2);
   const int64_t nslices = (n + mis + CT_SLICE - 1) / CT_SLICE;
@@ -294,7 +304,7 @@ int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, c
   const int64_t lim = (int64_t)num_sms() * 8;
   if (grid > lim) grid = lim;
   cudaError_t e = launch_pdl(ids_kernel, dim3((unsigned)grid), dim3(256), 0, s, (const uint32_t*)mk.fmask,
-                             (const uint32_t*)mk.meta, d_count, n, mis, sparse_den, ids);
+                             (const uint32_t*)mk.meta, d_count, n, mis, sparse_den, staged, ids);
   count_launch();
   if (e != cudaSuccess) return cuda_fail(e, "ids_kernel launch");
   return RA_OK;

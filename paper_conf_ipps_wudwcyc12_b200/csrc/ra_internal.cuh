@@ -145,7 +145,7 @@ int launch_gather(const uint32_t* ids, const int64_t* d_count, int64_t cap, cons
 // Sparse path without caller ids: the row ids from the select pass's SelMasks
 // (exits on the device when the count is dense).
 int launch_ids_from_masks(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count,
-                          int32_t sparse_den, uint32_t* ids, cudaStream_t s);
+                          int32_t sparse_den, int64_t staged, uint32_t* ids, cudaStream_t s);
 // Payload compaction from the select pass's SelMasks (compact.cu).
 int launch_compact(const int32_t* d_key, int64_t n, const SelMasks& mk, const int64_t* d_count, int64_t cap,
                    const GatherSpec& g, cudaStream_t s);

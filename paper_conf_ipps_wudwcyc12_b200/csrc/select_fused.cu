@@ -186,9 +186,12 @@ struct __align__(128) SelSmemT {
   uint32_t wtot[2][NW];                // [tile parity][warp] selected counts
   int32_t cnt[K];                      // tile aggregates
   int32_t start[K];                    // tile run start in the ring
+  int32_t rin[K];                      // ring rows of each tile (0 once past out_cap)
+  uint32_t past[2];                    // [tile parity] ROWS: the tile's ids land past out_cap
   int64_t n;
   uint32_t epoch;
   int32_t demand;  // oldest tile the compute warps are waiting to write (-1: none yet)
+  int32_t sat;     // ROWS: a resolved tile of this CTA ended at or past out_cap (monotone hint)
 };
 // A 40 KB ring (2 CTAs/SM).
 using SelSmem = SelSmemT<SEL_OUTRING>;
@@ -381,6 +384,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     S.n = n;
     S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);  // before any ticket: see the epoch note above
     S.demand = -1;
+    S.sat = 0;
     for (int s = 0; s < SEL_INSLOTS; ++s) {
       mbar_init(&S.full[s], 1);
       mbar_init(&S.empty[s], 1);
@@ -494,6 +498,10 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         my_prefix = g + S.cnt[k % K];
         if (lane == 0) {
           S.goff[k % K] = g;
+          // every later tile of this CTA has a larger index, so its offset is
+          // >= my_prefix: in ROWS mode with my_prefix >= out_cap none of its
+          // ids is written and the compute warps skip staging them
+          if (ROWS && my_prefix >= P.out_cap) st_relaxed_shared(&S.sat, 1);
           if (tp == ntiles - 1) {  // every tile has published (read the epoch): advance it
             *P.d_count = my_prefix;
             st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
@@ -596,6 +604,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       wtotal += (tot[q] & 0xFF) + ((tot[q] >> 8) & 0xFF) + ((tot[q] >> 16) & 0xFF) + (tot[q] >> 24);
     }
     if (lane == 0) S.wtot[i & 1][warp] = wtotal;
+    if (ROWS && tid == 0) S.past[i & 1] = (uint32_t)ld_relaxed_shared(&S.sat);  // one value for every thread
     PT_BEGIN(tb);
     compute_bar();  // B1: wtot visible; every warp is done with this tile's input slot
     PT_END(3, tb, tid == 0);
@@ -604,9 +613,11 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     const int32_t agg = (int32_t)__reduce_add_sync(0xffffffffu, wt);
     const int32_t wbase = (int32_t)__reduce_add_sync(0xffffffffu, lane < warp ? wt : 0u);
     if (ROWS && P.meta && lane == 0) P.meta[t * 12 + warp] = (uint32_t)wbase;
-    const bool ring_rows = !ROWS || P.rowids;  // ROWS without ids: placement only, no ring
+    // ROWS without ids, or with every id of this tile past out_cap: no ring rows
+    const bool ring_rows = !ROWS || (P.rowids && !S.past[i & 1]);
     const int32_t rows_in = ring_rows ? agg : 0;  // ring rows this tile needs
     if (tid == 0) {  // publish at once (before any wait below); hand the tile to the look-back warp
+      S.rin[i % K] = rows_in;
       mbar_arrive(&S.empty[slot]);  // input slot free: the producer refills it
       dev::st_relaxed_u64(P.status + t, FLAG_A | (tag << TAG_SHIFT) | (uint64_t)agg);
       S.cnt[i % K] = agg;
@@ -634,7 +645,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         break;
       }
       write_tile<ROWS, SM>(S, P, head, tid);
-      used -= ring_rows ? S.cnt[head % K] : 0;
+      used -= S.rin[head % K];
       ++head;
       forced = true;
     }
@@ -676,7 +687,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
     // ---- gather: tile i - LAG is due
     if (i - LAG >= head) {
       write_tile<ROWS, SM>(S, P, head, tid);
-      used -= ring_rows ? S.cnt[head % K] : 0;
+      used -= S.rin[head % K];
       ++head;
     }
   }

@@ -42,8 +42,8 @@ CAPTURES = {  # report -> (summary name, traffic key, command)
                     "python scripts/prof_driver.py multi 5 28 4  (2^28 int32, 4 outputs: .5 .5 .25 .25)"),
     "prof_sparse_sel": ("sparse_select_k1_s001_n28", "sparse_select_k1_s0.01_n28",
                         "python scripts/prof_driver.py sparse 5 28 1 0.01  (key pass of the sparse tuple SELECT)"),
-    "prof_sparse_ids": ("sparse_ids_k1_s001_n28", "sparse_ids_k1_s0.01_n28",
-                        "python scripts/prof_driver.py sparse 5 28 1 0.01  (ids_kernel: row ids from the order masks)"),
+    "prof_sparse_ids": ("sparse_ids_k1_s005_n28", "sparse_ids_k1_s0.05_n28",
+                        "python scripts/prof_driver.py sparse 5 28 1 0.05  (ids_kernel: the row ids past the n/32 the key pass staged, from the order masks)"),
     "prof_sparse_gather": ("sparse_gather_k1_s001_n28", "sparse_gather_k1_s0.01_n28",
                            "python scripts/prof_driver.py sparse 5 28 1 0.01  (gather_kernel: 3 int32 fields at the ids)"),
 }

@@ -110,7 +110,7 @@ def main():
         outs = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in chains]
         for _ in range(reps):
             R.select_multi(x, chains, outs=outs)
-    elif what == "sparse":  # f3 sparse path: 3 int32 fields at s=0.01 (ids_kernel + gather_kernel)
+    elif what == "sparse":  # f3 sparse path: 3 int32 fields, no caller ids (key pass + ids_kernel + gather_kernel)
         n = 1 << log2n
         x = torch.empty(n, dtype=torch.int32, device="cuda")
         ragen.int32_column_dev(2, x)

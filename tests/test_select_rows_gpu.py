@@ -142,7 +142,7 @@ def test_capacity_never_writes_past_cap(R, cap):
     assert (ids[cap:].cpu().numpy() == 0xABCDEF).all() and (out[cap:].cpu().numpy() == -9).all()
 
 
-@pytest.mark.parametrize("s", [0.03, 0.25, 0.6])
+@pytest.mark.parametrize("s", [0.03, 0.05, 0.1, 0.25, 0.6])
 @pytest.mark.parametrize("force_gather", [False, True])
 def test_both_payload_paths(R, s, force_gather, monkeypatch):
     """The device picks the id gather (sparse) or the streaming compaction
@@ -156,10 +156,39 @@ def test_both_payload_paths(R, s, force_gather, monkeypatch):
     key = ragen.int32_column(69, n)
     p4 = ragen.int32_column(70, n)
     preds = [("lt", t) for t in ragen.nested_thresholds(s, 1)]
-    for rowids in (True, False):  # without ids the sparse path rebuilds them from the masks (ids_kernel)
+    # without ids the sparse path takes the first n/32 from the key pass and
+    # rebuilds the rest from the masks (ids_kernel): s = .05 / .1 use both
+    for rowids in (True, False):
         check(R, key, preds, [p4, key], rowids=rowids)  # 4-byte fields only
         check(R, key, preds, [p4.astype(np.int64) * 5 - 7, p4], rowids=rowids)  # with an 8-byte field
         check(R, key, preds, [p4, key], offset=3, rowids=rowids)  # misaligned key view
+
+
+@pytest.mark.parametrize("cap", [0, 1, 5000, 20000, 60000])
+def test_capacity_without_ids_sparse(R, cap):
+    """No caller ids, sparse (count between n/32 and n/12): the key pass stages
+    min(out_cap, n/32) ids and ids_kernel the rest; the fields are exact up to
+    out_cap and nothing is written past it."""
+    n = 100 * 8192 + 77
+    key = ragen.int32_column(71, n)
+    p4 = ragen.int32_column(72, n)
+    preds = [("lt", t) for t in ragen.nested_thresholds(0.06, 1)]
+    exp_ids, (exp,) = oracle.select_rows(key, preds, [p4])
+    assert n // 32 < exp_ids.size < n // 12
+    kd, pd = torch.from_numpy(key).cuda(), torch.from_numpy(p4).cuda()
+    out = torch.full((cap + 64,), -9, dtype=torch.int32, device="cuda")
+    pl = (R.ra_payload * 1)()
+    pl[0].col, pl[0].out, pl[0].elem_bytes = pd.data_ptr(), out.data_ptr(), 4
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    wsb = R.ra_select_rows_workspace_bytes(n, 1)
+    ws = torch.zeros(wsb, dtype=torch.uint8, device="cuda")
+    R.ra_select_rows(kd.data_ptr(), n, R.make_preds(preds), 1, 0, pl, 1, cap, cnt.data_ptr(),
+                     ws.data_ptr(), wsb, int(torch.cuda.current_stream().cuda_stream))
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == exp_ids.size
+    m = min(cap, exp_ids.size)
+    assert np.array_equal(out[:m].cpu().numpy(), exp[:m])
+    assert (out[m:].cpu().numpy() == -9).all()
 
 
 def test_argument_errors(R):

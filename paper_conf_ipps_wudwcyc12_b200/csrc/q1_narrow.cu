@@ -8,10 +8,10 @@
 // price) raises the rows/s ceiling ~3.5x.  At 11 B/row the per-row arithmetic
 // becomes the limit, so the accumulation is restructured as well:
 //
-// q1n_kernel — persistent, two CTAs per SM, warp-specialised like the wide
-//   q1_tma_kernel: a producer warp streams 1024-row tiles of the six columns
-//   (six cp.async.bulk copies, 11 KB per tile) through a 4-stage
-//   shared-memory ring on mbarriers; 8 compute warps take 4 rows per thread
+// q1n_kernel — persistent, one CTA per SM, warp-specialised like the wide
+//   q1_tma_kernel: a producer warp streams 2048-row tiles of the six columns
+//   (six cp.async.bulk copies, 22 KB per tile) through a 4-stage
+//   shared-memory ring on mbarriers; 16 compute warps take 4 rows per thread
 //   per tile.  The domain checks and the SELECT of a thread's four rows run
 //   in SWAR form on the packed words (nrow4: per byte, bit 7 = out of
 //   domain), then each row is projected and added (nadd).  Instead of a predicated update of all 6 group slots per row
@@ -59,14 +59,24 @@ namespace {
 
 using namespace q1c;
 
-constexpr int QN_NT = 256;     // compute threads + 1 producer warp
+// One CTA of 16 compute warps per SM with a 4-stage ring of 2048-row tiles
+// (90 KB in flight per SM): measured 8% (SF10) / 5% (SF100) faster than two
+// CTAs of 8 warps with 1024-row tiles, and faster than 2 or 3 CTAs with more
+// warps and fewer stages (scripts/gpu_q1n_ab.sh, profiles/r02_q1n_ab.txt).
+#ifndef RA_Q1N_NT
+#define RA_Q1N_NT 512
+#endif
+constexpr int QN_NT = RA_Q1N_NT;  // compute threads (+ 1 producer warp)
 constexpr int QN_NW = QN_NT / 32;
-constexpr int QN_TILE = 1024;  // rows per tile (11 KB)
+constexpr int QN_TILE = 4 * QN_NT;  // rows per tile (2048: 22 KB)
 #ifndef RA_Q1N_STAGES
 #define RA_Q1N_STAGES 4
 #endif
 constexpr int QN_STAGES = RA_Q1N_STAGES;
-constexpr int QN_CTAS_PER_SM = 2;
+#ifndef RA_Q1N_CTAS
+#define RA_Q1N_CTAS 1
+#endif
+constexpr int QN_CTAS_PER_SM = RA_Q1N_CTAS;
 constexpr int QN_R = QN_TILE / QN_NT;  // 4 rows per thread per tile
 constexpr int QN_FLUSH_TILES = 256 / QN_R;
 static_assert(QN_R == 4, "the per-thread loads below take 4 rows");
@@ -75,7 +85,10 @@ static_assert(QN_R == 4, "the per-thread loads below take 4 rows");
 constexpr int NO_P = 0, NO_SD = 4 * QN_TILE, NO_Q = 6 * QN_TILE, NO_G = 8 * QN_TILE, NO_D = 9 * QN_TILE,
               NO_T = 10 * QN_TILE;
 constexpr int NSTAGE_BYTES = 11 * QN_TILE;
-constexpr int TRASH = NS;  // record index of unselected / out-of-domain rows
+// Record of unselected / out-of-domain rows.  (Predicating the reductions
+// instead: ptxas branches around each ATOMS, measured 1.5x slower.)
+constexpr int TRASH = NS;
+constexpr int NREC = NS + 1;
 
 struct QnParams {
   const uint16_t* sd;
@@ -96,9 +109,9 @@ struct QnParams {
 struct QnSmem {
   alignas(128) unsigned char stage[QN_STAGES][NSTAGE_BYTES];
 #if RA_Q1N_RED
-  uint32_t rec[NS + 1][7][QN_NT];  // [slot][field][thread]: thread-private records, lane-contiguous fields
+  uint32_t rec[NREC][7][QN_NT];  // [slot][field][thread]: thread-private records, lane-contiguous fields
 #else
-  uint4 rec[NS + 1][2][QN_NT];  // [slot][half][thread]: thread-private 32-byte records
+  uint4 rec[NREC][2][QN_NT];  // [slot][half][thread]: thread-private 32-byte records
 #endif
 #if RA_Q1N_WSLICE
   unsigned long long wsum[QN_NW][NS][6];  // per-warp sums: count, qty, price, disc, disc_price, charge
@@ -110,6 +123,12 @@ struct QnSmem {
   bool last;
 };
 constexpr size_t QN_SMEM = sizeof(QnSmem);
+
+struct QnRows {  // one thread's 4 rows of a tile
+  uint4 p;
+  uint2 sd, q;
+  uint32_t g, d, t;
+};
 static_assert(QN_SMEM <= 227 * 1024, "narrow Q1 kernel exceeds the shared-memory opt-in limit");
 
 __device__ __forceinline__ uint4 lds128(uint32_t a) {
@@ -299,7 +318,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
   }
   if (tid < QN_NT) {
 #pragma unroll
-    for (int s = 0; s <= NS; ++s) {
+    for (int s = 0; s < NREC; ++s) {
 #if RA_Q1N_RED
       for (int f = 0; f < 7; ++f) S.rec[s][f][tid] = 0u;
 #else
@@ -335,18 +354,30 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
     const uint32_t rec0 = dev::smem_u32(&S.rec[0][0][tid]);
     uint32_t status = 0, accg = 0, accn = 0;
     int i = 0, since = 0;
-    for (int64_t tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x, ++i) {
+    // the thread's 4 rows of tile i: stage -> registers, then the stage is released
+    auto load = [&](int i, QnRows& r) {
       const int s = i % QN_STAGES;
       dev::mbar_wait(&S.full[s], (i / QN_STAGES) & 1);
       const unsigned char* st = S.stage[s];
-      const uint4 p = *reinterpret_cast<const uint4*>(st + NO_P + 16 * tid);
-      const uint2 sd = *reinterpret_cast<const uint2*>(st + NO_SD + 8 * tid);
-      const uint2 q = *reinterpret_cast<const uint2*>(st + NO_Q + 8 * tid);
-      const uint32_t g = *reinterpret_cast<const uint32_t*>(st + NO_G + 4 * tid);
-      const uint32_t d = *reinterpret_cast<const uint32_t*>(st + NO_D + 4 * tid);
-      const uint32_t t = *reinterpret_cast<const uint32_t*>(st + NO_T + 4 * tid);
+      r.p = *reinterpret_cast<const uint4*>(st + NO_P + 16 * tid);
+      r.sd = *reinterpret_cast<const uint2*>(st + NO_SD + 8 * tid);
+      r.q = *reinterpret_cast<const uint2*>(st + NO_Q + 8 * tid);
+      r.g = *reinterpret_cast<const uint32_t*>(st + NO_G + 4 * tid);
+      r.d = *reinterpret_cast<const uint32_t*>(st + NO_D + 4 * tid);
+      r.t = *reinterpret_cast<const uint32_t*>(st + NO_T + 4 * tid);
       __syncwarp();
       if (lane == 0) dev::mbar_arrive(&S.empty[s]);  // the stage's values are in registers
+    };
+    // (Software-pipelining the stage loads — tile i+1 read before tile i is
+    // processed — measured 2-4% slower: the early barrier wait stalls the warp.
+    // Reading the rows from global memory instead of the TMA-staged tile,
+    // 1 or 2 tiles ahead: 35-40% slower, narrow LDGs cost more LSU cycles.)
+    for (int64_t tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x, ++i) {
+      QnRows cur;
+      load(i, cur);
+      const uint4 p = cur.p;
+      const uint2 sd = cur.sd, q = cur.q;
+      const uint32_t g = cur.g, d = cur.d, t = cur.t;
 #if RA_Q1N_SWAR
       nrow4(rec0, accg, accn, P.cutoff, sd, g, q, d, t, p);
 #elif RA_Q1N_PRMT  // byte i of g/d/t with one byte permute each (PRMT) instead of shift + mask
@@ -370,7 +401,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
       }
     }
     nflush(S, rec0);
-    // tail rows after the full tiles (< 1 per thread)
+    // tail rows after the full tiles (< 4 per thread)
     const int64_t tail0 = P.ntiles * QN_TILE;
     for (int64_t r = tail0 + (int64_t)blockIdx.x * QN_NT + tid; r < P.n; r += (int64_t)gridDim.x * QN_NT)
       nrow(rec0, status, P.cutoff, P.sd[r], P.g[r], P.q[r], P.d[r], P.t[r], P.p[r]);

@@ -1,6 +1,7 @@
+# narrow Q1 A/B: libra.so vs build/libra_$V.so variants (q1time: SF10 and SF100, CUDA events)
 mkdir -p gpurun_out
-NCU=/usr/local/cuda/bin/ncu
-$NCU --set full --import-source on --clock-control none -f -k regex:select_multi -s 2 -c 1 -o gpurun_out/prof_select_n30 python scripts/prof_driver.py select 3 30 > gpurun_out/ncu_n30.log 2>&1; echo n30 rc=$?
-( timeout -s KILL 300 python scripts/prof_driver.py q1time 20
-  RA_LIB_PATH=$PWD/build/libra_qs5.so timeout -s KILL 300 python scripts/prof_driver.py q1time 20
-  RA_LIB_PATH=$PWD/build/libra_qs3.so timeout -s KILL 300 python scripts/prof_driver.py q1time 20 ) 2>&1 | grep narrow | tee gpurun_out/q1n_stages.txt
+( for v in "" $VARIANTS; do
+  echo "== ${v:-libra.so}"
+  L=${v:+$PWD/build/libra_$v.so}
+  RA_LIB_PATH=$L timeout -s KILL 300 python scripts/prof_driver.py q1time 20 | grep narrow
+done ) 2>&1 | tee gpurun_out/q1n_ab.txt

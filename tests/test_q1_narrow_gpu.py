@@ -58,7 +58,7 @@ def assert_same(rows, exp):
             assert r[k] == e[k], (r["returnflag"], r["linestatus"], k, r[k], e[k])
 
 
-@pytest.mark.parametrize("n", [0, 1, 5, 1023, 1024, 1025, 4097, 100003, 1_000_000])
+@pytest.mark.parametrize("n", [0, 1, 5, 1023, 1024, 1025, 2047, 2048, 2049, 4097, 100003, 1_000_000])
 def test_encode_matches_numpy_and_q1_matches_oracle(R, n):
     cols = ragen.lineitem(51 + n, n, 20000)
     enc, st = R.q1_encode(dev(cols))

@@ -57,6 +57,9 @@ for M, sel in cases:
         _, cnt = R.select_multi(x, ch, outs=outs[:M])
     f = t(fused)
     kept = sum(int(c) for c in cnt.cpu().tolist()[:M])
+    if os.environ.get("MS_FUSED_ONLY"):
+        print(f"{M}  {str(sel):24s} {f:8.4f}", flush=True)
+        continue
     sp = t(lambda: [R.select_chain(x, ch[o], out=outs[o]) for o in range(M)])
     gbs = (4 * n + 4 * kept) / (f * 1e-3) / 1e9
     print(f"{M}  {str(sel):24s} {f:8.4f} {gbs:7.0f} {gbs / PEAK:6.3f}  | {sp:10.4f} {sp / f:10.3f}", flush=True)

@@ -2,6 +2,7 @@
 #include <cub/cub.cuh>
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
 
 struct LessThan {
   int32_t t;
@@ -16,12 +17,13 @@ __global__ void fill(int32_t* x, int64_t n, uint64_t seed) {
   }
 }
 
-int main() {
-  int64_t n = 1ll << 28;
+int main(int argc, char** argv) {
+  const int lg = argc > 1 ? atoi(argv[1]) : 28;
+  int64_t n = 1ll << lg;
   int32_t *x, *out; int* cnt;
   cudaMalloc(&x, n * 4); cudaMalloc(&out, n * 4); cudaMalloc(&cnt, 8);
   fill<<<1184, 256>>>(x, n, 7);
-  for (double s : {0.25, 0.5, 0.9, 0.01}) {
+  for (double s : {0.01, 0.1, 0.25, 0.5, 0.75, 0.9}) {
     LessThan op{(int32_t)(-2147483648.0 + s * 4294967296.0)};
     size_t tb = 0; void* tmp = nullptr;
     cub::DeviceSelect::If(tmp, tb, x, out, cnt, (int)n, op);
@@ -33,7 +35,7 @@ int main() {
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b); ms /= 20;
     int c; cudaMemcpy(&c, cnt, 4, cudaMemcpyDeviceToHost);
-    printf("cub select s=%.2f: %.4f ms  count %d  alg GB/s %.1f  (%s)\n", s, ms, c, (4.0 * n + 4.0 * c) / ms / 1e6,
+    printf("cub select 2^%d s=%.2f: %.4f ms  count %d  alg GB/s %.1f  (%s)\n", lg, s, ms, c, (4.0 * n + 4.0 * c) / ms / 1e6,
            cudaGetErrorString(cudaGetLastError()));
     cudaFree(tmp);
   }

@@ -248,6 +248,9 @@ __device__ __forceinline__ void nrow4(uint32_t rec0, uint32_t& accg, uint32_t& a
 //   count <= 256 (<< 16 -> < 2^25), disc <= 25600 < 2^16, qty < 2^16 * 2^8,
 //   price <= (2^24-1) * 2^8 < 2^32, dp>>16 < 2^15 * 2^8, dp&0xffff < 2^16 * 2^8,
 //   tax*(dp>>16) < 100 * 2^15 * 2^8 < 2^30, tax*(dp&0xffff) < 100 * 2^16 * 2^8 < 2^31.
+// Summed over a warp's 32 lanes: count <= 2^13, disc < 2^21, qty < 2^29,
+// dp>>16 < 2^28, dp&0xffff < 2^29 fit one 32-bit REDUX; price and the tax*dp
+// halves need the 16-bit split (warp_sum32).
 // A CTA takes <= 2^24 rows (launch_q1_narrow), so its charge sum stays below
 // 200 * 100 * 2^24 * 2^24 < 2^63 and every CTA sum fits 64 bits.
 // Warp sum of 32-bit values as an exact 64-bit value: REDUX on the 16-bit
@@ -270,9 +273,12 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
     const uint4 a = lds128(ra), b = lds128(ra + REC_HALF);
 #endif
     if (!__any_sync(0xffffffffu, (a.x | a.y | a.z | a.w | b.x | b.y | b.z) != 0u)) continue;  // warp-uniform
-    const unsigned long long cnt = warp_sum32(a.x >> 16), disc = warp_sum32(a.x & 0xFFFFu);
-    const unsigned long long q = warp_sum32(a.y), p = warp_sum32(a.z);
-    const unsigned long long dph = warp_sum32(a.w), dpl = warp_sum32(b.x);
+    // fields whose 32 lanes sum below 2^32 (bounds above) take one REDUX, the
+    // others (price, tax*dp halves) two
+    const unsigned long long cnt = __reduce_add_sync(0xffffffffu, a.x >> 16);
+    const unsigned long long disc = __reduce_add_sync(0xffffffffu, a.x & 0xFFFFu);
+    const unsigned long long q = __reduce_add_sync(0xffffffffu, a.y), p = warp_sum32(a.z);
+    const unsigned long long dph = __reduce_add_sync(0xffffffffu, a.w), dpl = __reduce_add_sync(0xffffffffu, b.x);
     const unsigned long long chh = warp_sum32(b.y), chl = warp_sum32(b.z);
     if (lane == 0) {
 #if RA_Q1N_WSLICE  // this warp's own sums: plain 64-bit adds (64-bit shared atomics are CAS loops)
@@ -400,8 +406,9 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
         since = 0;
       }
     }
-    nflush(S, rec0);
-    // tail rows after the full tiles (< 4 per thread)
+    // tail rows after the full tiles (< QN_TILE rows: at most 4 per thread), into
+    // the same records: fewer than 64 tiles since the last flush, so at most
+    // 4 * 63 + 4 = 256 rows per record between flushes (nflush's bound)
     const int64_t tail0 = P.ntiles * QN_TILE;
     for (int64_t r = tail0 + (int64_t)blockIdx.x * QN_NT + tid; r < P.n; r += (int64_t)gridDim.x * QN_NT)
       nrow(rec0, status, P.cutoff, P.sd[r], P.g[r], P.q[r], P.d[r], P.t[r], P.p[r]);

@@ -254,13 +254,14 @@ int q1_fission_generic(const void* const* cols, const char* const* names, const 
   }
   const int S = n_streams;
   int result = RA_OK;
-  // zero each stream's running partial and its Q1 ticket word (the region
+  // zero each stream's running partial and its Q1 ticket, status and grid
+  // accumulators (the region
   // layout moves with chunk_rows)
   for (int s = 0; s < S && result == RA_OK; ++s) {
     char* base = (char*)d_ws + (size_t)s * R.total;
     cudaStream_t st = (cudaStream_t)streams[s];
     cudaError_t e = cudaMemsetAsync(base + R.part, 0, sizeof(ra_q1_partial), st);
-    if (e == cudaSuccess) e = cudaMemsetAsync(base + R.ws, 0, 256, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(base + R.ws, 0, q1_ws_clear_bytes(), st);
     if (e != cudaSuccess) result = cuda_fail(e, "cudaMemsetAsync(q1 fission partials)");
   }
   const int64_t C = (n + chunk_rows - 1) / chunk_rows;

@@ -12,7 +12,7 @@ namespace q1c {
 constexpr int NS = RA_Q1_GROUPS;
 constexpr int Q1_MAX_GRID = 148 * 8;
 
-struct Q1Block {
+struct Q1Block {  // (sizes the ABI's Q1 workspace: ra_q1_workspace_bytes)
   uint32_t status;
   uint32_t _pad;
   uint64_t v[NS][8];  // count, qty, price, disc, dp_lo, dp_hi, ch_lo, ch_hi
@@ -57,12 +57,37 @@ __device__ __forceinline__ void warp_sum_u128(uint64_t& lo, uint64_t& hi) {
   }
 }
 
-// Reduction: warp (shuffles) -> CTA (smem) -> grid (last CTA, 128-bit fold).
-// Called by every thread of the CTA; warps >= NW (a producer warp) only join
-// the barriers.  s_w: [NW][NS][8] shared scratch.
+// Grid accumulators (in the workspace; zero between launches): per slot
+// ACC_K u64 — count, qty, price, disc, then the 128-bit disc_price and charge
+// sums as three limbs each (bits 0-31, bits 32-63, bits 64-127 of every CTA's
+// value).  Every CTA adds its partial with 64-bit atomics (RED), so no add
+// overflows: <= Q1_MAX_GRID 32-bit limbs sum below 2^43, and the 64-bit
+// fields' grid sums stay < 2^63 through SF100 (C11).  The last CTA in reads
+// and clears them in ONE round of atomic exchanges and composes the
+// ra_q1_partial: a walk over per-CTA partials cost ~6 us of dependent L2
+// round trips at the end of every launch (stamped with %globaltimer,
+// scripts/q1n_times.py).  Workspace header: u32 CTA ticket @0, u32 status @4.
+constexpr int ACC_K = 10;
+constexpr int ACC_OFFSET = 256;  // bytes from the workspace start
+
+template <typename Params>
+__device__ __forceinline__ void acc_add(const Params& P, int s, int k, uint64_t v) {
+  if (v) atomicAdd(P.acc + s * ACC_K + k, (unsigned long long)v);  // result unused: RED
+}
+// which: 0 = disc_price, 1 = charge
+template <typename Params>
+__device__ __forceinline__ void acc_add128(const Params& P, int s, int which, uint64_t lo, uint64_t hi) {
+  acc_add(P, s, 4 + 3 * which, lo & 0xFFFFFFFFull);
+  acc_add(P, s, 5 + 3 * which, lo >> 32);
+  acc_add(P, s, 6 + 3 * which, hi);
+}
+
 template <typename Params>
 __device__ __forceinline__ void publish_and_fold(const Params& P, bool* s_last);
 
+// Reduction: warp (shuffles) -> CTA (smem) -> grid (atomic accumulators, last
+// CTA composes).  Called by every thread of the CTA; warps >= NW (a producer
+// warp) only join the barriers.  s_w: [NW][NS][8] shared scratch.
 template <int NW, typename Params>
 __device__ __forceinline__ void reduce_and_fold(const Acc& A, const Params& P, uint64_t (*s_w)[NS][8],
                                                 uint32_t* s_status, bool* s_last) {
@@ -93,7 +118,6 @@ __device__ __forceinline__ void reduce_and_fold(const Acc& A, const Params& P, u
     }
   }
   __syncthreads();
-  Q1Block* mine = P.blocks + blockIdx.x;
   if (threadIdx.x < NS * 4) {  // (slot, field pair)
     const int s = threadIdx.x >> 2, f = threadIdx.x & 3;
     if (f < 2) {  // count/qty or price/disc: 64-bit
@@ -102,44 +126,48 @@ __device__ __forceinline__ void reduce_and_fold(const Acc& A, const Params& P, u
         a += s_w[w][s][2 * f];
         b += s_w[w][s][2 * f + 1];
       }
-      mine->v[s][2 * f] = a;
-      mine->v[s][2 * f + 1] = b;
+      acc_add(P, s, 2 * f, a);
+      acc_add(P, s, 2 * f + 1, b);
     } else {  // dp or ch: 128-bit
       uint64_t lo = 0, hi = 0;
       for (int w = 0; w < NW; ++w) add128(lo, hi, s_w[w][s][2 * f], s_w[w][s][2 * f + 1]);
-      mine->v[s][2 * f] = lo;
-      mine->v[s][2 * f + 1] = hi;
+      acc_add128(P, s, f - 2, lo, hi);
     }
   }
-  if (threadIdx.x == 0) mine->status = *s_status;
+  if (threadIdx.x == 0 && *s_status) atomicOr(P.counter + 1, *s_status);
   publish_and_fold(P, s_last);
 }
 
-// After this CTA wrote its Q1Block: ticket; the last CTA to arrive folds all
-// CTA partials into *P.out (128-bit where needed).  Called by every thread.
+// After this CTA added its partial: ticket; the last CTA to arrive reads and
+// clears the accumulators and writes *P.out (128-bit where needed).  Called
+// by every thread (blockDim.x > NS * ACC_K).
 template <typename Params>
 __device__ __forceinline__ void publish_and_fold(const Params& P, bool* s_last) {
-  __threadfence();
+  __shared__ unsigned long long s_acc[NS * ACC_K];
+  __shared__ uint32_t s_st;
+  __threadfence();  // this thread's accumulator adds happen before the ticket
   __syncthreads();
   if (threadIdx.x == 0) *s_last = (atomicAdd(P.counter, 1u) == gridDim.x - 1);
   __syncthreads();
   if (!*s_last) return;
 
-  // ---- last CTA: fold all CTA partials (128-bit where needed)
+  // ---- last CTA: every other CTA's adds are performed; read + clear at once
   __threadfence();
-  const int nb = gridDim.x;
+  if (threadIdx.x < NS * ACC_K) s_acc[threadIdx.x] = atomicExch(P.acc + threadIdx.x, 0ull);
+  if (threadIdx.x == NS * ACC_K) s_st = atomicExch(P.counter + 1, 0u);
+  __syncthreads();
   if (threadIdx.x < NS * 4) {
     const int s = threadIdx.x >> 2, f = threadIdx.x & 3;
-    uint64_t a = 0, b = 0;
-    for (int i = 0; i < nb; ++i) {
-      const uint64_t x = __ldcg(&P.blocks[i].v[s][2 * f]);
-      const uint64_t y = __ldcg(&P.blocks[i].v[s][2 * f + 1]);
-      if (f < 2) {
-        a += x;
-        b += y;
-      } else {
-        add128(a, b, x, y);
-      }
+    const unsigned long long* v = s_acc + s * ACC_K;
+    uint64_t a, b;
+    if (f < 2) {
+      a = v[2 * f];
+      b = v[2 * f + 1];
+    } else {  // limbs (bits 0-31, 32-63, 64-127) -> 128-bit
+      const unsigned long long* l = v + 4 + 3 * (f - 2);
+      a = l[0];
+      b = l[2];
+      add128(a, b, l[1] << 32, l[1] >> 32);
     }
     ra_q1_group* G = &P.out->group[s];
     if (P.accumulate) {  // exact: 64-bit sums stay < 2^63 through SF100 (C11), 128-bit ones carry
@@ -164,9 +192,8 @@ __device__ __forceinline__ void publish_and_fold(const Params& P, bool* s_last) 
       G->sum_charge_lo = a;
       G->sum_charge_hi = (int64_t)b;
     }
-  } else if (threadIdx.x == 32) {
-    uint32_t st = 0;
-    for (int i = 0; i < nb; ++i) st |= __ldcg(&P.blocks[i].status);
+  } else if (threadIdx.x == NS * 4) {
+    const uint32_t st = s_st;
     P.out->status = P.accumulate ? (P.out->status | st) : st;
     P.out->n_groups = NS;
     P.out->rows = P.accumulate ? P.out->rows + (uint64_t)P.n : (uint64_t)P.n;

@@ -61,8 +61,8 @@ struct Q1Params {
   int32_t cutoff;
   ra_q1_partial* out;
   int accumulate;  // add into *out (chunks of one query under fission) instead of overwriting
-  Q1Block* blocks;
-  uint32_t* counter;
+  unsigned long long* acc;  // grid accumulators [NS][ACC_K] (q1_common.cuh)
+  uint32_t* counter;        // [0] CTA ticket, [1] status
 };
 
 // Per-row SELECT + domain checks + group slot + PROJECT.  Returns the slot
@@ -451,6 +451,9 @@ int64_t common_head(const ra_lineitem& c, int64_t n, int flag_align) {
 }  // namespace
 
 size_t q1_ws_bytes() { return 256 + (size_t)Q1_MAX_GRID * sizeof(Q1Block); }
+size_t q1_ws_clear_bytes() { return ACC_OFFSET + sizeof(unsigned long long) * NS * ACC_K; }
+static_assert(ACC_OFFSET + sizeof(unsigned long long) * NS * ACC_K <= 256 + Q1_MAX_GRID * sizeof(Q1Block),
+              "accumulators inside the Q1 workspace");
 
 int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_partial, void* d_ws,
               size_t ws_bytes, cudaStream_t s, int accumulate) {
@@ -468,7 +471,7 @@ int launch_q1(const ra_lineitem& c, int64_t n, int32_t cutoff, ra_q1_partial* d_
   P.out = d_partial;
   P.accumulate = accumulate;
   P.counter = (uint32_t*)d_ws;
-  P.blocks = (Q1Block*)((char*)d_ws + 256);
+  P.acc = (unsigned long long*)((char*)d_ws + ACC_OFFSET);
   const int dev = current_device();
   // per-thread 64-bit sums stay exact while rows/thread <= 2^17
   const int64_t sms = num_sms();

@@ -38,6 +38,17 @@
 
 #include <stdio.h>
 
+#ifdef RA_Q1N_TIMES  // diagnostics build: per-CTA %globaltimer stamps (scripts/q1n_times.py)
+__device__ unsigned long long g_qn_t[1184][16];
+#define QN_T(k)                                                  \
+  do {                                                           \
+    if (threadIdx.x == 0) {                                      \
+      unsigned long long t_;                                     \
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));     \
+      g_qn_t[blockIdx.x][k] = t_;                                \
+    }                                                            \
+  } while (0)
+#endif
 #include "q1_common.cuh"
 
 namespace ra {
@@ -102,8 +113,8 @@ struct QnParams {
   int32_t cutoff;
   ra_q1_partial* out;
   int accumulate;
-  Q1Block* blocks;
-  uint32_t* counter;
+  unsigned long long* acc;  // grid accumulators [NS][ACC_K] (q1_common.cuh)
+  uint32_t* counter;        // [0] CTA ticket, [1] status
 };
 
 struct QnSmem {
@@ -308,8 +319,21 @@ __device__ __forceinline__ void nflush(QnSmem& S, uint32_t rec0) {
   }
 }
 
+#ifndef RA_Q1N_TIMES
+#define QN_T(k)
+#endif
+
 __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const QnParams P) {
+  QN_T(0);
   dev::grid_dep_wait();  // launch_pdl: the previous kernel's writes (e.g. a running partial) are visible
+  QN_T(1);
+#ifdef RA_Q1N_TIMES
+  if (threadIdx.x == 0) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    g_qn_t[blockIdx.x][7] = smid;
+  }
+#endif
   extern __shared__ __align__(128) unsigned char qn_smem_raw[];
   QnSmem& S = *reinterpret_cast<QnSmem*>(qn_smem_raw);
   const int tid = threadIdx.x;
@@ -335,6 +359,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
   for (int i = tid; i < (int)(sizeof(S.wsum) / 8); i += blockDim.x) reinterpret_cast<unsigned long long*>(S.wsum)[i] = 0ull;
   if (tid == 0) S.status = 0;
   __syncthreads();
+  QN_T(2);
 
   if (warp == QN_NW) {
     // ---------------- producer warp: one elected lane issues the bulk copies
@@ -406,6 +431,7 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
         since = 0;
       }
     }
+    QN_T(3);
     // tail rows after the full tiles (< QN_TILE rows: at most 4 per thread), into
     // the same records: fewer than 64 tiles since the last flush, so at most
     // 4 * 63 + 4 = 256 rows per record between flushes (nflush's bound)
@@ -413,12 +439,13 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
     for (int64_t r = tail0 + (int64_t)blockIdx.x * QN_NT + tid; r < P.n; r += (int64_t)gridDim.x * QN_NT)
       nrow(rec0, status, P.cutoff, P.sd[r], P.g[r], P.q[r], P.d[r], P.t[r], P.p[r]);
     nflush(S, rec0);
+    QN_T(4);
     status |= (accg ? 1u : 0u) | (accn ? 2u : 0u);
     if (status) atomicOr(&S.status, status);
   }
-  // CTA partial -> P.blocks[blockIdx]; the last CTA folds all of them
+  // CTA partial -> the grid accumulators; the last CTA composes the result
   __syncthreads();
-  if (tid < NS * 6) {  // CTA sums (of the warps' sums) -> P.blocks[blockIdx]: v = {cnt, qty, price, disc, dp lo/hi, ch lo/hi}
+  if (tid < NS * 6) {  // CTA sums (of the warps' sums) -> the grid accumulators: cnt, qty, price, disc, dp, ch
     const int sl = tid / 6, f = tid % 6;
 #if RA_Q1N_WSLICE
     unsigned long long v = 0;
@@ -426,13 +453,16 @@ __global__ void __launch_bounds__(QN_NT + 32, QN_CTAS_PER_SM) q1n_kernel(const Q
 #else
     const unsigned long long v = S.wsum[sl][f];
 #endif
-    Q1Block* mine = P.blocks + blockIdx.x;
-    static constexpr int DST[6] = {0, 1, 2, 3, 4, 6};
-    mine->v[sl][DST[f]] = v;
-    if (f >= 4) mine->v[sl][DST[f] + 1] = 0;
+    if (f < 4) {
+      acc_add(P, sl, f, v);
+    } else {
+      acc_add128(P, sl, f - 4, v, 0ull);
+    }
   }
-  if (tid == 0) P.blocks[blockIdx.x].status = S.status;
+  if (tid == 0 && S.status) atomicOr(P.counter + 1, S.status);
+  QN_T(5);
   publish_and_fold(P, &S.last);
+  QN_T(6);
 }
 
 // ------------------------------------------------------------- encoder
@@ -486,7 +516,7 @@ int launch_q1_narrow(const ra_lineitem_narrow& c, int64_t n, int32_t cutoff, ra_
   P.out = d_partial;
   P.accumulate = accumulate;
   P.counter = (uint32_t*)d_ws;
-  P.blocks = (Q1Block*)((char*)d_ws + 256);
+  P.acc = (unsigned long long*)((char*)d_ws + ACC_OFFSET);
   const int a = device_once(g_qn_attr, current_device(), [] {
     cudaError_t e = cudaFuncSetAttribute(q1n_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)QN_SMEM);
     return e != cudaSuccess ? cuda_fail(e, "q1n_kernel smem attribute") : 1;
@@ -526,3 +556,10 @@ int launch_q1_encode(const ra_lineitem& in, int64_t n, const ra_lineitem_narrow_
 }
 
 }  // namespace ra
+
+#ifdef RA_Q1N_TIMES
+extern "C" __attribute__((visibility("default"))) int raqn_times(unsigned long long* out) {
+  cudaDeviceSynchronize();
+  return (int)cudaMemcpyFromSymbol(out, g_qn_t, sizeof(g_qn_t));
+}
+#endif

@@ -161,6 +161,9 @@ int select_chain_impl(const int32_t* d_in, int64_t n, const ra_pred* h_preds, in
 int launch_q1(const ra_lineitem& cols, int64_t n, int32_t cutoff, ra_q1_partial* d_partial,
               void* d_ws, size_t ws_bytes, cudaStream_t s, int accumulate = 0);
 size_t q1_ws_bytes();
+// Leading bytes of a Q1 workspace that carry state between launches (ticket,
+// status, grid accumulators): zero them to start a workspace afresh.
+size_t q1_ws_clear_bytes();
 // Narrow Q1 (f4): same workspace and partial as launch_q1; columns 16-B aligned.
 int launch_q1_narrow(const ra_lineitem_narrow& cols, int64_t n, int32_t cutoff, ra_q1_partial* d_partial,
                      void* d_ws, cudaStream_t s, int accumulate = 0);

@@ -39,6 +39,22 @@
 
 #include "ra_internal.cuh"
 
+#ifdef RA_MO_TIMES  // diagnostics build: per-CTA %globaltimer stamps (scripts/mo_times.py)
+__device__ unsigned long long g_mo_t[2048][16];
+#define MO_T(k)                                              \
+  do {                                                       \
+    unsigned long long t_;                                   \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));   \
+    g_mo_t[blockIdx.x][k] = t_;                              \
+  } while (0)
+extern "C" __attribute__((visibility("default"))) int ramo_times(unsigned long long* out) {
+  cudaDeviceSynchronize();
+  return (int)cudaMemcpyFromSymbol(out, g_mo_t, sizeof(g_mo_t));
+}
+#else
+#define MO_T(k)
+#endif
+
 namespace ra {
 
 namespace {
@@ -402,8 +418,15 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
   SM& S = *reinterpret_cast<SM*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
+  if (tid == 0) MO_T(0);
   dev::grid_dep_wait();  // programmatic dependent launch: previous grid's writes visible
   if (tid == 0) {
+    MO_T(1);
+#ifdef RA_MO_TIMES
+    unsigned smid_;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid_));
+    g_mo_t[blockIdx.x][8] = smid_;
+#endif
     int64_t n = P.n;
     if (P.d_n) {
       const int64_t dn = dev::ld_relaxed_s64(P.d_n);
@@ -433,6 +456,7 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  if (tid == 0) MO_T(2);
   const int64_t n = S.n;
   const int64_t nv = n + P.mis;
   const int64_t ntiles = n > 0 ? (nv + TILE - 1) / TILE : 0;
@@ -458,6 +482,7 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
         if (j >= INSLOTS) MWAIT(&S.empty[s], (uint32_t)((j / INSLOTS - 1) & 1), 1, (int)j);
         if (RA_MO_LATE_TICKET && ends == 0) cur = (int64_t)atomicAdd(P.ticket, 1ull);
         if (cur >= ntiles) {  // one end marker per compute group (ntiles + e: e = 0 is the true end)
+          if (ends == 0) MO_T(3);
           S.tile_of[s] = ntiles + ends;
           mbar_arrive(&S.full[s]);
           if (++ends == NG) break;
@@ -570,6 +595,7 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
     // the CTA's last look-back warp out joins the grid-wide epilogue:
     // last CTA out resets the ticket; at a tag wrap it clears every status word
     if (lane == 0 && atomicAdd(&S.lb_done, 1) == NLB - 1) {
+      MO_T(6);
       __threadfence();
       if (atomicAdd(&P.hdr[H_DONE], 1u) == gridDim.x - 1) {
         *P.ticket = 0ull;
@@ -598,7 +624,10 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
     constexpr int NWR = C::NWR, WT = 32 * NWR, WU = RA_MO_WU;
     for (int k = 0;; ++k) {
       MWAIT(&S.placed[k % K], (uint32_t)((k / K) & 1), 4, (int)k);
-      if (S.tidx[k % K] < 0) break;
+      if (S.tidx[k % K] < 0) {
+        if (wt == 0) MO_T(7);
+        break;
+      }
       MWAIT(&S.scattered[k % K], (uint32_t)((k / K) & 1), 5, (int)k);
       int32_t base = S.start[k % K];
       PROF_T0(t_wr);
@@ -641,9 +670,11 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
     const int slot = i % INSLOTS;
     PROF_T0(t_it);
     MWAIT(&S.full[slot], (uint32_t)((i / INSLOTS) & 1), 6, (int)i);
+    if (i == 0 && gtid == 0) MO_T(4);
     const int64_t t = S.tile_of[slot];
     if (t >= ntiles) {
       if (t == ntiles && gtid == 0) {  // the true end: tile i is this CTA's tile count
+        MO_T(5);
         if (i >= K) MWAIT(&S.written[i % K], (uint32_t)(((i / K) - 1) & 1), 7, (int)i);
         S.tidx[i % K] = -1;
         st_release_shared(&S.end_tile, i);

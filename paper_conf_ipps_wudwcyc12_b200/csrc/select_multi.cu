@@ -99,7 +99,13 @@ constexpr int H_EPOCH = 0, H_DONE = 4, H_HWM = 6;
 #define RA_MO_D1 0
 #endif
 #ifndef RA_MO_IN_KB
-#define RA_MO_IN_KB 96  // input ring per CTA
+#define RA_MO_IN_KB 96  // input ring per CTA, one output
+#endif
+#ifndef RA_MO_IN_KB2
+// two outputs: 2 input slots, the rest of shared memory to the ring of
+// selected rows (3 slots were 15% slower when both outputs keep ~half the rows
+// with overlapping predicates: the ring filled and placements queued behind it)
+#define RA_MO_IN_KB2 64
 #endif
 constexpr int NG = RA_MO_NG;
 constexpr int GW = 8;                         // warps per compute group
@@ -132,7 +138,7 @@ struct Cfg {
   static constexpr int WROWS = TILE / GW;            // contiguous rows per compute warp
   static constexpr int NPK = VEC / 4;                // packed 8-bit count words per lane per output
   static constexpr int W = (M + 1) / 2;              // status words per tile
-  static constexpr int INSLOTS = (M <= 2 ? RA_MO_IN_KB : RA_MO_IN_KB34) * 1024 / (TILE * 4);
+  static constexpr int INSLOTS = (M == 1 ? RA_MO_IN_KB : M == 2 ? RA_MO_IN_KB2 : RA_MO_IN_KB34) * 1024 / (TILE * 4);
   static constexpr int D1 = RA_MO_D1 > 0 ? RA_MO_D1 : (M == 1 ? 2 : 1);
   static constexpr int NWR = M <= 2 ? RA_MO_NWR : RA_MO_NWR34;           // writer warps
   static constexpr int BLOCK = 32 * (NCW + NLB + 1 + NWR);

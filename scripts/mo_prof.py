@@ -24,10 +24,11 @@ ragen.int32_column_dev(2, x)
 outs = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
 buf = (ctypes.c_ulonglong * 64)()
 CASES = {"m1": [(1, 0.01), (1, 0.25)], "dense": [(2, 0.9), (4, 0.9), (4, 0.5)],
-         "m2pair": [(2, 0.5), (2, "comp")]}.get(
+         "m2pair": [(2, 0.5), (2, "comp")], "m4bench": [(4, "bench4")]}.get(
     os.environ.get("MO_PROF_CASES", ""), [(1, 0.01), (1, 0.5), (2, 0.5), (2, 0.9), (3, 0.01)])
 for M, s in CASES:
     ch = ([[("lt", 0)], [("ge", 0)]] if s == "comp"  # complementary pair
+          else [[("lt", 0)], [("gt", -(2**30)), ("lt", 2**30)], [("ge", 2**30)], [("lt", -(2**30))]] if s == "bench4"
           else [[("lt", ragen.nested_thresholds(s, 1)[0])]] * M)
     for _ in range(3):
         R.select_multi(x, ch, outs=outs[:M])

@@ -447,20 +447,29 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
     S.end_tile = 0x7fffffff;
     S.lb_done = 0;
     for (int o = 0; o < M; ++o) S.pfx[o] = 0;
-    for (int s = 0; s < INSLOTS; ++s) {
-      mbar_init(&S.full[s], 1);
-      mbar_init(&S.empty[s], 1);
-    }
-    for (int q = 0; q < Q; ++q) mbar_init(&S.winfull[q], 1);
-    for (int s = 0; s < K; ++s) {
-      mbar_init(&S.counted[s], 1);
-      mbar_init(&S.placed[s], 1);
-      mbar_init(&S.scattered[s], RA_MO_SCAT_ARRIVALS);
-      mbar_init(&S.written[s], 1);
-      mbar_init(&S.allocd[s], 1);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  // mbarriers initialised in parallel, one thread each (a serial init by one
+  // thread was ~0.5 us of every launch's ramp)
+  static_assert(2 * INSLOTS <= 32 && Q <= 32 && K <= 32, "init lanes");
+  if (tid >= 32 && tid < 32 + 2 * INSLOTS) mbar_init(tid & 1 ? &S.empty[(tid - 32) >> 1] : &S.full[(tid - 32) >> 1], 1);
+  if (tid >= 64 && tid < 64 + Q) mbar_init(&S.winfull[tid - 64], 1);
+  if (tid >= 96 && tid < 96 + K) {
+    const int s = tid - 96;
+    mbar_init(&S.counted[s], 1);
+    mbar_init(&S.placed[s], 1);
+    mbar_init(&S.scattered[s], RA_MO_SCAT_ARRIVALS);
+    mbar_init(&S.written[s], 1);
+    mbar_init(&S.allocd[s], 1);
+  }
+  if ((tid >= 32 && tid < 32 + 2 * INSLOTS) || (tid >= 64 && tid < 64 + Q) || (tid >= 96 && tid < 96 + K))
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+#ifndef RA_MO_LATE_TICKET
+#define RA_MO_LATE_TICKET 0
+#endif
+  // the producer's first ticket is drawn before the barrier: its round trip
+  // overlaps the init (the previous launch reset the ticket; grid_dep_wait above)
+  int64_t first_ticket = 0;
+  if (!RA_MO_LATE_TICKET && warp == PRWARP && lane == 0) first_ticket = (int64_t)atomicAdd(P.ticket, 1ull);
   __syncthreads();
   if (tid == 0) MO_T(2);
   const int64_t n = S.n;
@@ -477,11 +486,8 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
 #endif
   if (warp == PRWARP) {
     // ========================= producer: partition + load =====================
-#ifndef RA_MO_LATE_TICKET
-#define RA_MO_LATE_TICKET 0
-#endif
     if (lane == 0) {
-      int64_t cur = RA_MO_LATE_TICKET ? 0 : (int64_t)atomicAdd(P.ticket, 1ull);
+      int64_t cur = first_ticket;
       int ends = 0;
       for (int j = 0;; ++j) {
         const int s = j % INSLOTS;

@@ -58,8 +58,8 @@
 // 768-word slots copied one tile late: 0.230 ms.  1 CTA/SM with deeper input
 // rings is far slower (0.34 ms) — scripts/sel_variants.sh + scripts/gpu_selvar.sh.)
 //
-// Status words carry a 28-bit launch epoch (header word bumped by the last
-// tile), so stale words of earlier launches read as "not ready": no per-call
+// Status words carry a 28-bit launch epoch (header word advanced by the last
+// CTA to finish, so every CTA of a launch reads the same value), so stale words of earlier launches read as "not ready": no per-call
 // memset and no second kernel.  The ticket counter is reset by the last CTA to
 // finish.  The launch before the tag wraps to 0 clears every status word the
 // workspace has held (header high-water mark), so tags never alias.
@@ -382,7 +382,7 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
       n = dn < n ? (dn < 0 ? 0 : dn) : n;
     }
     S.n = n;
-    S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);  // before any ticket: see the epoch note above
+    S.epoch = ld_acquire_u32(&P.hdr[H_EPOCH]);  // advanced only by the last CTA out (epoch note above)
     S.demand = -1;
     S.sat = 0;
     for (int s = 0; s < SEL_INSLOTS; ++s) {
@@ -502,16 +502,14 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
           // >= my_prefix: in ROWS mode with my_prefix >= out_cap none of its
           // ids is written and the compute warps skip staging them
           if (ROWS && my_prefix >= P.out_cap) st_relaxed_shared(&S.sat, 1);
-          if (tp == ntiles - 1) {  // every tile has published (read the epoch): advance it
-            *P.d_count = my_prefix;
-            st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
-          }
+          if (tp == ntiles - 1) *P.d_count = my_prefix;  // every tile has published
           mbar_arrive(&S.placed[k % K]);
         }
         __syncwarp();
       }
     }
-    // last CTA out resets the ticket counter for the next launch
+    // last CTA out resets the ticket counter for the next launch and advances
+    // the epoch (after every CTA of this launch read it: one tag per launch)
     if (lane == 0) {
       __threadfence();
       if (atomicAdd(&P.hdr[H_DONE], 1u) == gridDim.x - 1) {
@@ -526,8 +524,9 @@ __global__ void __launch_bounds__(BLOCK, 2) select_fused_kernel(const SelParams 
         uint64_t* hwm = reinterpret_cast<uint64_t*>(P.hdr + H_HWM);
         uint64_t h = *hwm;
         if ((uint64_t)ntiles > h) *hwm = h = (uint64_t)ntiles;
-        if (ntiles > 0 && ((S.epoch + 1) & TAG_MASK) == 0)
+        if (((S.epoch + 1) & TAG_MASK) == 0)
           for (uint64_t w = 0; w < h; ++w) P.status[w] = 0ull;
+        st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
       }
     }
     return;

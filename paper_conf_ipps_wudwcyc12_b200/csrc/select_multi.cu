@@ -592,10 +592,9 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
           S.goff[k % K][o] = g;
           S.pfx[o] = g + S.cnt[k % K][o];
         }
-        if (tc == ntiles - 1) {  // the last tile: every tile has published; totals, then the epoch
+        if (tc == ntiles - 1) {  // the last tile: every tile has published; the totals
 #pragma unroll
           for (int o = 0; o < M; ++o) *P.d_count[o] = S.pfx[o];
-          st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
         }
         PROF_LAT(18, S.t_count[k % K]);
         PROF_STAMP(S.t_placed[k % K]);
@@ -604,8 +603,10 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
       }
       __syncwarp();
     }
-    // the CTA's last look-back warp out joins the grid-wide epilogue:
-    // last CTA out resets the ticket; at a tag wrap it clears every status word
+    // the CTA's last look-back warp out joins the grid-wide epilogue: the last
+    // CTA out resets the ticket, at a tag wrap clears every status word, and
+    // advances the epoch — after every CTA of this launch read it, so all of
+    // them (also a late one that drew no tile) used the same tag
     if (lane == 0 && atomicAdd(&S.lb_done, 1) == NLB - 1) {
       MO_T(6);
       __threadfence();
@@ -619,8 +620,9 @@ __global__ void __launch_bounds__(Cfg<M>::BLOCK, 1) select_multi_kernel(const __
         uint64_t* hwm = reinterpret_cast<uint64_t*>(P.hdr + H_HWM);
         uint64_t h = *hwm;
         if ((uint64_t)(ntiles * W) > h) *hwm = h = (uint64_t)(ntiles * W);
-        if (ntiles > 0 && ((S.epoch + 1) & TAG_MASK) == 0)
+        if (((S.epoch + 1) & TAG_MASK) == 0)
           for (uint64_t w = 0; w < h; ++w) P.status[w] = 0ull;
+        st_release_u32(&P.hdr[H_EPOCH], S.epoch + 1);
       }
     }
     return;

@@ -252,6 +252,39 @@ def test_epoch_tag_wrap_clears_stale_status_words(R, base):
     assert int(hdr32[0].item()) == (1 << 28) + 2 and int(hdr64[3].item()) == hw
 
 
+@pytest.mark.parametrize("big", [False, True])
+def test_epoch_advances_once_per_launch_even_without_tiles(R, big):
+    """The epoch is advanced by the last CTA out (so every CTA of a launch,
+    also one that drew no tile, uses the same tag), once per launch — also for
+    n = 0.  A wrap that falls on an empty launch still clears the stale words:
+    planted "tag 0" words must not read as published in the next launch.
+    big: above 2^21 rows (multi-output pass), else the single-output pass."""
+    n_big = (1 << 21) + 40 * 8192 + 5 if big else 40 * 8192 + 5
+    ws = torch.zeros(R.ra_select_workspace_bytes(n_big, 1, 1), dtype=torch.uint8, device="cuda")
+    hw = min((n_big + 8191) // 8192 + 7, (ws.numel() - 256) // 8)  # >= the big launch's tiles
+    words = ws[256:].view(torch.int64)
+    hdr32, hdr64 = ws[:256].view(torch.int32), ws[:256].view(torch.int64)
+    words[:hw] = (1 << 62) | 1000          # stale "tag 0" words with bogus aggregates
+    hdr32[0] = (1 << 28) - 1               # the next launch is the last before the wrap
+    hdr64[3] = hw
+    preds = [("lt", 0)]
+    sh = int(torch.cuda.current_stream().cuda_stream)
+    P = R.make_preds(preds)
+    empty = torch.empty(1, dtype=torch.int32, device="cuda")
+    cnt = torch.full((1,), -1, dtype=torch.int64, device="cuda")
+    R.ra_select_chain(empty.data_ptr(), 0, P, 1, 1, empty.data_ptr(), 0, cnt.data_ptr(), ws.data_ptr(), ws.numel(), sh)
+    torch.cuda.synchronize()
+    assert int(cnt.item()) == 0 and int(hdr32[0].item()) == 1 << 28
+    x = torch.from_numpy(ragen.int32_column(7, n_big)).cuda()
+    out = torch.empty(n_big, dtype=torch.int32, device="cuda")
+    R.ra_select_chain(x.data_ptr(), n_big, P, 1, 1, out.data_ptr(), n_big, cnt.data_ptr(), ws.data_ptr(), ws.numel(), sh)
+    torch.cuda.synchronize()
+    exp = oracle.select(x.cpu().numpy(), preds)
+    assert int(cnt.item()) == exp.size
+    np.testing.assert_array_equal(out[:exp.size].cpu().numpy(), exp)
+    assert int(hdr32[0].item()) == (1 << 28) + 1
+
+
 def test_select_rows_workspace_reuse_across_sizes(R):
     """Tuple SELECT keeps its order masks and staged ids at the END of the
     workspace: a later call with larger n on the same (bigger) workspace never

@@ -680,7 +680,9 @@ def extras(args, D, torch, R, x, preds, kept, chain_ms):
     a1 = (x1.data_ptr(), n1, P1, 1, 1, o1.data_ptr(), n1, c1.data_ptr(), ws1.data_ptr(), ws1_b, sh)
     ms1, _ = timed(torch, D, lambda i, kernel_done=False: R.ra_select_chain(*a1), 200, 10)
     ex["select_1m"] = {"us_per_call": ms1 * 1e3, "rows_per_s": n1 / (ms1 * 1e-3), "kept": int(c1.item()),
-                       "note": "configs[0]; 6 MiB L2-resident, back-to-back stream launches"}
+                       "note": "configs[0]; 6 MiB L2-resident; back-to-back C-ABI calls from Python (the "
+                               "ctypes call itself takes ~6-8 us on the host, so this can be host-bound); "
+                               "graph_us_per_call = the same calls replayed from a CUDA graph (device time)"}
     try:  # d1: CUDA-graph replay of 100 captured C-ABI calls (launch latency off the host)
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g):

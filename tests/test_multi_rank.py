@@ -125,3 +125,24 @@ def test_exchange_counts_host_scan():
     """exchange_counts on host tensors uses plain integer code for the scan."""
     assert rdist.exclusive_offsets([]) == []
     assert rdist.exclusive_offsets([2**40, 1, 0]) == [0, 2**40, 2**40 + 1]
+
+
+def test_bench_reference_arm_under_torchrun_two_ranks():
+    """`bench.py --impl reference` launched the driver's way for N=2 (torchrun,
+    127.0.0.1): rank 0 alone times the oracle and prints one JSON line with
+    impl=reference, the other rank exits 0 without work.  CPU only."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", str(29500 + os.getpid() % 2000),
+           os.path.join(root, "bench.py"), "--impl", "reference", "--gpus", "2", "--steps", "1", "--warmup", "1",
+           "--rows-log2", "18"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=300, cwd=root)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["unit"] == "rows/s" and d["value"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["cpu_baseline"]["kind"] == "oracle"

@@ -206,6 +206,28 @@ def test_full_size_four_outputs(R):
         np.testing.assert_array_equal(o[:int(c)].cpu().numpy(), e)
 
 
+@pytest.mark.parametrize("pair", ["identical", "nested", "complementary"])
+def test_two_outputs_ring_pressure(R, pair):
+    """Two outputs keeping ~half (or all) of 2^24 rows each with overlapping
+    predicates: the regime where the ring of selected rows runs full (2 input
+    slots for M = 2, placements on demand), and the two outputs' offsets move
+    in lockstep.  Full comparison with the oracle, 4 launches on one workspace."""
+    n = 1 << 24
+    x = torch.empty(n, dtype=torch.int32, device="cuda")
+    ragen.int32_column_dev(11, x)
+    chains = {"identical": [[("lt", 0)], [("lt", 0)]],
+              "nested": [[("lt", 2**30)], [("ge", -(2**31))]],
+              "complementary": [[("lt", 0)], [("ge", 0)]]}[pair]
+    exp = oracle.select_multi(x.cpu().numpy(), chains)
+    outs = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(2)]
+    for _ in range(4):
+        _, cnt = R.select_multi(x, chains, outs=outs)
+        torch.cuda.synchronize()
+        for o, c, e in zip(outs, cnt.cpu().tolist(), exp):
+            assert int(c) == e.size
+            np.testing.assert_array_equal(o[:int(c)].cpu().numpy(), e)
+
+
 def test_full_size_bench_config(R):
     """bench.py's f2 leg at full size (2^28 device-generated rows, seed 2, the
     bench's two chains), full comparison of both outputs with the oracle."""

@@ -202,6 +202,10 @@ struct __align__(128) MoSmem : MoFixed<M> {
   static constexpr int RING = ring_ints<M>();
   alignas(128) int32_t ring[RING];  // runs start at multiples of 32 rows (128-B aligned)
 };
+// the producer ends with one marker per compute group in consecutive slots,
+// and a group that takes a marker releases no slot: every marker needs its own
+static_assert(Cfg<1>::INSLOTS >= NG && Cfg<2>::INSLOTS >= NG && Cfg<3>::INSLOTS >= NG && Cfg<4>::INSLOTS >= NG,
+              "input slots >= compute groups");
 static_assert(MoSmem<1>::RING >= Cfg<1>::TILE && MoSmem<2>::RING >= 2 * Cfg<2>::TILE &&
                   MoSmem<3>::RING >= 3 * Cfg<3>::TILE && MoSmem<4>::RING >= 4 * Cfg<4>::TILE,
               "a tile's M runs must always fit an empty ring");

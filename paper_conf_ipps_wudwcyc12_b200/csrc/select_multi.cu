@@ -129,7 +129,9 @@ constexpr int SMEM_BUDGET = 232448;           // max dynamic shared memory per C
 
 #ifndef RA_MO_VEC34
 #define RA_MO_VEC34 8     // M = 3, 4: int4 vectors per compute lane per tile
-#define RA_MO_IN_KB34 64  //           input ring per CTA
+#endif
+#ifndef RA_MO_IN_KB34
+#define RA_MO_IN_KB34 64  // M = 3, 4: input ring per CTA
 #endif
 template <int M>
 struct Cfg {
